@@ -1,0 +1,341 @@
+#!/usr/bin/env python
+"""Benchmark: 8x8 Reversi playouts/s on B200 (BASELINE.json metric, configs[1]).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+
+One "step" = one pass of the playout hot path over one
+batch of BASELINE configs[1]: 4096 synthetic mid-game positions x 256 random
+playouts, inputs resident in HBM, launched through mcts_playouts_async. N>1:
+one process per GPU (torchrun), every rank runs its own batch with distinct
+playout streams (leaf_id_base = rank * 4096): weak scaling, no collective on
+the data path. The block-parallel search (configs[2] shape, a1-a11 incl. the
+NCCL root-stats allreduce at N>1) and the leaf-parallel comparison (configs[3])
+are reported in the "search" / "leaf_search" objects of the same line.
+
+Prints ONE JSON line on rank 0. See DESIGN.md §8 for every field.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_LEAVES, N_PER_LEAF, GEN_SEED, LMIN, LMAX = 4096, 256, 2, 20, 40
+PLAYOUT_SEED = 2
+SEARCH_TREES, SEARCH_THREADS, SEARCH_MS = 1184, 128, 500.0
+LEAF_THREADS = 16384
+METRIC = "8x8 Reversi playouts/sec at 1/2/4/8 B200; win% vs CPU-oracle MCTS"
+# Algorithmic 32-bit integer operations per ply (one move decision) of the
+# shift-mask method, DESIGN.md §6 op model (movegen 2x8x24 incl. the final
+# shift + empty mask, flip 8x26, pick 30, Philox 96/4, loop 8).
+ALG_OPS_PER_PLY = 440
+
+
+def clocks_sampler(path):
+    try:
+        f = open(path, "w")
+        p = subprocess.Popen(
+            ["nvidia-smi", "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,"
+             "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+            stdout=f, stderr=subprocess.DEVNULL)
+        return p, f
+    except Exception:
+        return None, None
+
+
+def clocks_summary(path, gpu_index):
+    rows = []
+    try:
+        for line in open(path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 9 and parts[0] == str(gpu_index):
+                rows.append(parts)
+    except Exception:
+        pass
+    if not rows:
+        return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+    sm = sorted(float(r[1]) for r in rows)
+    names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+    reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
+    return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": float(rows[0][2]), "reasons": reasons,
+            "samples": len(rows)}
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def reference_arm(args, rank):
+    """--impl reference: the CPU oracle as it stands, on this box's host cores."""
+    if rank != 0:
+        return
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    leaves = oracle.gen_positions(GEN_SEED, N_LEAVES, LMIN, LMAX)
+    chunk = 64  # leaves per step: a bounded sample of the configs[1] batch
+
+    def step(i):
+        a = (i * chunk) % N_LEAVES
+        return oracle.playouts(leaves[a:a + chunk], N_PER_LEAF, PLAYOUT_SEED, leaf_id_base=a,
+                               nthreads=cores)
+
+    for i in range(args.warmup):
+        step(i)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        step(args.warmup + i)
+    dt = time.perf_counter() - t0
+    value = args.steps * chunk * N_PER_LEAF / dt
+    sample = f"{chunk} leaves x {N_PER_LEAF} playouts of configs[1] per step"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "playouts/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": "configs[1]: 4096 mid-game positions x 256 playouts (sampled)",
+                   "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "playouts/s", "cores": cores, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": "playouts/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def cpu_baseline(budget_s=12.0):
+    """The oracle timed on the host cores on a bounded sample of configs[1]."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    leaves = oracle.gen_positions(GEN_SEED, N_LEAVES, LMIN, LMAX)
+    done, t0 = 0, time.perf_counter()
+    while done < N_LEAVES and time.perf_counter() - t0 < budget_s:
+        oracle.playouts(leaves[done:done + 128], N_PER_LEAF, PLAYOUT_SEED, leaf_id_base=done,
+                        nthreads=cores)
+        done += 128
+    dt = time.perf_counter() - t0
+    return {"value": done * N_PER_LEAF / dt, "unit": "playouts/s", "cores": cores, "kind": "oracle",
+            "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
+    ap.add_argument("--no-search", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--search-ms", type=float, default=SEARCH_MS)
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return reference_arm(args, rank)
+    if args.warmup < 3:
+        args.warmup = 3
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_rockis11_b200 as pkg
+    from paper_conf_ipps_rockis11_b200 import device as dev
+    from paper_conf_ipps_rockis11_b200.distributed import merge_root_stats
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x: int) -> int:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.int64, device="cuda")
+        dist.all_reduce(t)
+        return int(t.item())
+
+    m = pkg.Mcts(c_uct=1.0, scheme="block", device=local)
+    stream = torch.cuda.current_stream()
+    leaf_base = rank * N_LEAVES
+    d_leaves = dev.gen_positions(m, GEN_SEED, N_LEAVES, LMIN, LMAX)
+    d_out = dev.empty_wdl(N_LEAVES)
+    d_plies = torch.zeros(1, dtype=torch.int64, device="cuda")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+
+    def step():
+        m.playouts_async(d_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, leaf_base,
+                         d_out.data_ptr(), d_plies.data_ptr(), stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    d_plies.zero_()
+
+    clk_path = os.path.join(tempfile.gettempdir(), f"bench_clocks_{os.getpid()}.csv")
+    sampler, sampler_f = clocks_sampler(clk_path)
+    time.sleep(0.3)
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        flush.zero_()  # L2 flush outside the timed events
+        starts[i].record(stream)
+        step()
+        ends[i].record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    kernel_ms = sum(s.elapsed_time(e) for s, e in zip(starts, ends))
+    plies_local = int(d_plies.item())
+    t_ms = max_over_ranks(kernel_ms)
+    plies_total = sum_over_ranks(plies_local)
+    playouts_total = world * args.steps * N_LEAVES * N_PER_LEAF
+    value = playouts_total / (t_ms / 1e3)
+    ms_per_step = t_ms / args.steps
+
+    # ---- end to end through the C ABI with host buffers (H2D + kernel + D2H)
+    from paper_conf_ipps_rockis11_b200.positions import own_opp  # noqa: F401
+    h_leaves = torch.empty((N_LEAVES, 3), dtype=torch.int64).pin_memory()
+    h_leaves.copy_(d_leaves.cpu())
+    h_out = torch.empty((N_LEAVES, 3), dtype=torch.int32).pin_memory()
+    e2e_steps = max(3, args.steps // 2)
+    for _ in range(2):
+        m.playouts_host_ptr(h_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, h_out.data_ptr())
+    barrier()
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        m.playouts_host_ptr(h_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, h_out.data_ptr())
+    e2e_s = max_over_ranks(time.perf_counter() - t0)
+    barrier()
+    e2e_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_s
+
+    # ---- block-parallel search, configs[2] shape, time mode, + root allreduce
+    search = None
+    leaf_search = None
+    launches = args.steps  # one playouts_kernel per timed step
+    if not args.no_search:
+        root = pkg.position(*pkg.OPENING)
+        sstats = torch.zeros(198, dtype=torch.int64, device="cuda")
+        m.search_async(root, 0, 50.0, SEARCH_TREES, SEARCH_THREADS, 1000, rank * SEARCH_TREES,
+                       sstats.data_ptr(), stream)  # warm-up (pool + ln table)
+        torch.cuda.synchronize()
+        barrier()
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        m.search_async(root, 0, args.search_ms, SEARCH_TREES, SEARCH_THREADS, 1000,
+                       rank * SEARCH_TREES, sstats.data_ptr(), stream)
+        with torch.cuda.stream(stream):
+            merge_root_stats(sstats)
+        s1.record(stream)
+        torch.cuda.synchronize()
+        s_ms = max_over_ranks(s0.elapsed_time(s1))
+        st = sstats.cpu().numpy()
+        search = {
+            "workload": f"configs[2] shape: {SEARCH_TREES} trees x {SEARCH_THREADS} threads per GPU, "
+                        f"{args.search_ms:.0f} ms time mode, opening root, C=1.0",
+            "playouts_per_s": float(st[195]) / (s_ms / 1e3), "ms": s_ms,
+            "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
+            "plies_per_s": float(st[197]) / (s_ms / 1e3),
+            "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
+        }
+        ml = pkg.Mcts(c_uct=1.0, scheme="leaf", device=local)
+        lstats = torch.zeros(198, dtype=torch.int64, device="cuda")
+        ml.search_async(root, 0, 20.0, 1, LEAF_THREADS, 1000, rank, lstats.data_ptr(), stream)
+        torch.cuda.synchronize()
+        s0.record(stream)
+        ml.search_async(root, 0, args.search_ms, 1, LEAF_THREADS, 1000, rank, lstats.data_ptr(), stream)
+        with torch.cuda.stream(stream):
+            merge_root_stats(lstats)
+        s1.record(stream)
+        torch.cuda.synchronize()
+        l_ms = max_over_ranks(s0.elapsed_time(s1))
+        lt = lstats.cpu().numpy()
+        leaf_search = {
+            "workload": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch per GPU, "
+                        f"{args.search_ms:.0f} ms",
+            "playouts_per_s": float(lt[195]) / (l_ms / 1e3), "ms": l_ms,
+            "iterations": float(lt[196]) / world, "best_move": int(pkg.best_move(lt)),
+        }
+        ml.close()
+
+    if sampler is not None:
+        sampler.terminate()
+        sampler.wait()
+        sampler_f.close()
+    clocks = clocks_summary(clk_path, local)
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peaks = measured_peaks()
+    sm_max = peaks.get("sm_max_mhz", 1965.0)
+    peak_ops = 148 * 4 * 32 * sm_max * 1e6  # thread-instruction issue slots / s
+    kern_s = kernel_ms / 1e3 / args.steps
+    plies_per_launch = plies_local / args.steps
+    achieved = plies_per_launch * ALG_OPS_PER_PLY / kern_s
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))
+        traffic = prof.get("dram_bytes_per_launch")
+    except Exception:
+        pass
+    line = {
+        "metric": METRIC, "value": value, "unit": "playouts/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic",
+        "config": {"workload": "configs[1]: 4096 synthetic mid-game positions (seed 2, 20-40 random "
+                               "plies) x 256 random playouts per GPU",
+                   "global_batch": world * N_LEAVES * N_PER_LEAF,
+                   "parallelism": f"leaf-range x{world} (weak)",
+                   "l2": "flushed between steps (256 MiB write outside the timed events)"},
+        "plies_per_s": plies_total / (t_ms / 1e3),
+        "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak_ops / 1e9,
+                     "unit": "Gop/s", "frac": achieved / peak_ops, "traffic": traffic,
+                     "ops_per_ply": ALG_OPS_PER_PLY, "plies_per_launch": plies_per_launch,
+                     "peak_basis": f"issue slots 148 SM x 4 SMSP x 32 lanes x {sm_max:.0f} MHz "
+                                   "(MEASURED_PEAKS.json sm_max_mhz), DESIGN.md §6"},
+        "e2e": {"value": e2e_value, "unit": "playouts/s",
+                "h2d_bytes_per_step": N_LEAVES * 24, "d2h_bytes_per_step": N_LEAVES * 12 + 8,
+                "api": "mcts_playouts (host buffers, pinned)"},
+        "gpu_launches": launches,
+        "clocks": clocks,
+        "search": search, "leaf_search": leaf_search,
+    }
+    if not args.no_cpu and world == 1:
+        try:
+            line["cpu_baseline"] = cpu_baseline()
+        except Exception as e:  # the oracle is optional on the bench path
+            line["cpu_baseline"] = {"error": str(e)}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -505,7 +505,11 @@ int64_t orc_uct_tree(const orc_position* root, uint32_t unit, uint64_t iteration
 // with attempt + 1.
 void orc_gen_positions(uint64_t seed, uint32_t n, uint32_t lmin, uint32_t lmax, orc_position* out) {
   for (uint32_t p = 0; p < n; ++p) {
-    for (uint32_t attempt = 0;; ++attempt) {
+    // lmax <= 50 keeps >= 10 empty squares, so a non-terminal result is found
+    // after a few attempts; the cap only guards against misuse (result: opening).
+    out[p].black = 0x0000000810000000ULL; out[p].white = 0x0000001008000000ULL;
+    out[p].to_move = 0; out[p].reserved = 0;
+    for (uint32_t attempt = 0; attempt < (1u << 16); ++attempt) {
       uint32_t span = lmax - lmin + 1;
       uint32_t L = lmin + (uint32_t)(((uint64_t)rng_word(seed, p, 0xFFFFFFFFu, attempt, 0) * span) >> 32);
       uint64_t me = 0x0000000810000000ULL, op = 0x0000001008000000ULL;  // black, white

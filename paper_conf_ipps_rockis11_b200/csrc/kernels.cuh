@@ -1,0 +1,363 @@
+// kernels.cuh — the sm_100a kernels of the hot path.
+//
+//   playouts_kernel      a1-a6: batched random playouts, warp ballot W/D/L
+//   block_search_kernel  a1-a10: block-parallel UCT, one tree per CTA
+//                        (PAPER.md L294-L311), root merge fused at the end
+//   leaf_search_kernel   a12: leaf-parallel UCT, one tree, the whole grid
+//                        simulates from the same leaf
+//   ln_table_kernel      lnT[k] = RN(ln(k*unit)) for the UCB term (R9)
+//   gen_positions_kernel synthetic input recipe
+#pragma once
+#include <cstdint>
+#include "reversi_device.cuh"
+#include "ln_device.cuh"
+#include "tree_device.cuh"
+
+namespace mcts_dev {
+
+struct DevPosition {  // layout of mcts_position
+  u64 black, white;
+  u32 to_move, reserved;
+};
+
+struct WdlOut {  // layout of mcts_wdl
+  u32 wins, draws, losses;
+};
+
+__device__ __forceinline__ u64 globaltimer_ns() {
+  u64 t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// ---------------------------------------------------------------------------
+// Batched playouts. Thread g plays playout j = g mod n_per_leaf of leaf
+// g / n_per_leaf (leaf-major, so the 32 lanes of a warp usually share a leaf
+// and finish within a ply or two of each other). Outcomes are reduced per
+// (warp, leaf) with match_any + ballot + popc and added with one atomic per
+// counter; the ply count with one atomic per warp.
+// ---------------------------------------------------------------------------
+constexpr int kPlayoutThreads = 128;
+
+__global__ void __launch_bounds__(kPlayoutThreads)
+playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
+                u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out) {
+  const u64 g = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  const u64 total = (u64)n_leaves * n_per_leaf;
+  const bool active = g < total;
+  u32 leaf = 0xFFFFFFFFu, j = 0;
+  int r = 2;
+  u32 plies = 0;
+  if (active) {
+    leaf = (u32)(g / n_per_leaf);
+    j = (u32)(g - (u64)leaf * n_per_leaf);
+    const DevPosition p = leaves[leaf];
+    const u64 own = p.to_move ? p.white : p.black;
+    const u64 opp = p.to_move ? p.black : p.white;
+    r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, &plies);
+  }
+  const int lane = threadIdx.x & 31;
+  const u32 grp = __match_any_sync(kFull, leaf);
+  const u32 wins = __popc(__ballot_sync(kFull, r == 1) & grp);
+  const u32 draws = __popc(__ballot_sync(kFull, r == 0) & grp);
+  const u32 losses = __popc(__ballot_sync(kFull, r == -1) & grp);
+  if (active && lane == __ffs(grp) - 1) {
+    if (wins) atomicAdd(&out[leaf].wins, wins);
+    if (draws) atomicAdd(&out[leaf].draws, draws);
+    if (losses) atomicAdd(&out[leaf].losses, losses);
+  }
+  if (plies_out) {
+    const u32 s = __reduce_add_sync(kFull, plies);
+    if (lane == 0 && s) atomicAdd(plies_out, (unsigned long long)s);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Block-parallel UCT: CTA t owns tree t. Per iteration
+// warp 0 selects + expands (warp-cooperative UCB argmax), every thread plays
+// one playout from the new leaf (c0 = tree id, c1 = iteration, c2 = thread),
+// warps reduce outcomes with ballot/popc, warp 0 backpropagates. No host
+// round trip and no inter-CTA communication until the fused root merge.
+// ---------------------------------------------------------------------------
+struct SearchArgs {
+  DevPosition root;
+  uint2 key;
+  double C;
+  const double* lnT;
+  long long* stats;      // MCTS_STATS_LEN int64 (accumulated)
+  const u64* t0;         // device timestamp written before the launch (time mode)
+  u64 budget_ns;         // 0 = iteration mode
+  u32 max_iterations;    // iteration budget, or the time-mode cap
+  u32 tree_id_base;
+  u32 unit;              // playouts per iteration per tree
+  int* error;            // set on a watchdog bailout
+};
+
+constexpr int kSearchThreadsMax = 1024;
+
+template <int MAX_THREADS, int MIN_BLOCKS>
+__global__ void __launch_bounds__(MAX_THREADS, MIN_BLOCKS)
+block_search_kernel(TreePool T, SearchArgs a) {
+  __shared__ u32 path[kMaxPath];
+  __shared__ u64 s_own, s_opp;
+  __shared__ u32 s_term, s_stop, s_slot_used;
+  __shared__ u32 s_w[32], s_d[32];
+  __shared__ int s_depth;
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nwarps = blockDim.x >> 5;
+  const u32 tree = blockIdx.x;
+  const size_t base = (size_t)tree * T.slot_cap;
+  const u32 c0 = a.tree_id_base + tree;
+  const u32 unit = blockDim.x;
+  const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
+
+  if (tid == 0) {
+    const u64 own = a.root.to_move ? a.root.white : a.root.black;
+    const u64 opp = a.root.to_move ? a.root.black : a.root.white;
+    init_node(T, base, own, opp, 0xFFu);
+    s_slot_used = 1;
+  }
+  __syncthreads();
+
+  u32 plies = 0;
+  u32 it = 0;
+  if (!meta_term(T.meta[base])) {
+    for (;; ++it) {
+      if (warp == 0) {
+        u32 stop = 0;
+        if (lane == 0) {
+          stop = it >= a.max_iterations;
+          if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
+        }
+        stop = __shfl_sync(kFull, stop, 0);
+        if (!stop) {
+          const LeafInfo L = select_expand(T, base, path, &s_slot_used, a.lnT, unit, a.C, lane);
+          if (lane == 0) {
+            s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth;
+          }
+        }
+        if (lane == 0) s_stop = stop;
+      }
+      __syncthreads();
+      if (s_stop) break;
+      int r;
+      if (s_term) {
+        const int x = __popcll(s_own), y = __popcll(s_opp);
+        r = (x > y) - (x < y);
+      } else {
+        r = playout(s_own, s_opp, a.key, c0, it, (u32)tid, &plies);
+      }
+      const u32 bw = __popc(__ballot_sync(kFull, r == 1));
+      const u32 bd = __popc(__ballot_sync(kFull, r == 0));
+      if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
+      __syncthreads();
+      if (warp == 0) {
+        u32 W = lane < nwarps ? s_w[lane] : 0u;
+        u32 D = lane < nwarps ? s_d[lane] : 0u;
+        W = __reduce_add_sync(kFull, W);
+        D = __reduce_add_sync(kFull, D);
+        backprop(T, base, path, s_depth, W, D, unit - W - D, lane);
+      }
+    }
+  }
+  // fused per-GPU root merge (a10) + ply count
+  const u32 bp = __reduce_add_sync(kFull, plies);
+  if (lane == 0) s_w[warp] = bp;
+  __syncthreads();
+  if (warp == 0) {
+    unsigned long long P = lane < nwarps ? s_w[lane] : 0u;
+    for (int off = 16; off > 0; off >>= 1) P += __shfl_xor_sync(kFull, P, off);
+    if (lane == 0 && P) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, P);
+    merge_root(T, base, unit, it, a.stats, lane);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Leaf-parallel UCT: one tree; every thread of the grid
+// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree.
+// One gather/release barrier per iteration: CTAs add their counts and arrive,
+// CTA 0 waits for all arrivals, backpropagates, selects the next leaf and
+// releases the grid by bumping a generation word. All CTAs are co-resident
+// (cooperative launch); spins carry a watchdog so a fault cannot hang the GPU.
+// ---------------------------------------------------------------------------
+struct LeafSync {
+  u64 own, opp;
+  u32 term, stop;
+  u32 gen;          // released iteration + 1
+  u32 arrive;       // cumulative CTA arrivals
+  u32 wd[2][2];     // per-iteration-parity wins, draws
+};
+
+__device__ __forceinline__ u32 ld_acquire(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(u32* p, u32 v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+constexpr u64 kWatchdogNs = 120ULL * 1000000000ULL;
+
+__global__ void __launch_bounds__(128)
+leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
+  __shared__ u32 path[kMaxPath];
+  __shared__ u32 s_slot_used;
+  __shared__ int s_depth;
+  __shared__ u32 s_go;
+  __shared__ u32 s_w[4], s_d[4];
+  __shared__ u64 s_own, s_opp;
+  __shared__ u32 s_term;
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const u32 G = gridDim.x;
+  const bool leader_cta = blockIdx.x == 0;
+  const u32 unit = a.unit;
+  const u64 start = globaltimer_ns();
+  const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
+
+  if (leader_cta && tid == 0) {
+    const u64 own = a.root.to_move ? a.root.white : a.root.black;
+    const u64 opp = a.root.to_move ? a.root.black : a.root.white;
+    init_node(T, 0, own, opp, 0xFFu);
+    s_slot_used = 1;
+  }
+  __syncthreads();
+  const bool root_term = leader_cta ? meta_term(T.meta[0]) : false;
+
+  u32 plies = 0;
+  u32 it = 0;
+  for (;; ++it) {
+    if (leader_cta && warp == 0) {
+      if (it > 0) {
+        // wait for all CTAs of iteration it-1, then backprop
+        if (lane == 0) {
+          const u32 want = G * it;
+          while (ld_acquire(&S->arrive) < want) {
+            if (globaltimer_ns() - start > kWatchdogNs) { atomicExch(a.error, 1); break; }
+          }
+        }
+        __syncwarp();
+        const u32 par = (it - 1) & 1u;
+        u32 W = 0, D = 0;
+        if (lane == 0) {
+          W = *((volatile u32*)&S->wd[par][0]);
+          D = *((volatile u32*)&S->wd[par][1]);
+          S->wd[par][0] = 0; S->wd[par][1] = 0;
+        }
+        W = __shfl_sync(kFull, W, 0);
+        D = __shfl_sync(kFull, D, 0);
+        backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
+      }
+      u32 stop = 0;
+      if (lane == 0) {
+        stop = root_term || it >= a.max_iterations || *((volatile int*)a.error) != 0;
+        if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
+      }
+      stop = __shfl_sync(kFull, stop, 0);
+      if (!stop) {
+        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
+        if (lane == 0) {
+          s_depth = L.depth;
+          S->own = L.own; S->opp = L.opp; S->term = L.term;
+        }
+      }
+      if (lane == 0) {
+        S->stop = stop;
+        __threadfence();
+        st_release(&S->gen, it + 1);
+      }
+    }
+    // every CTA: wait for the release of iteration `it`
+    if (tid == 0) {
+      while (ld_acquire(&S->gen) < it + 1) {
+        if (globaltimer_ns() - start > kWatchdogNs) { atomicExch(a.error, 1); break; }
+      }
+      s_go = *((volatile u32*)&S->stop) == 0u && *((volatile int*)a.error) == 0;
+      s_own = *((volatile u64*)&S->own);
+      s_opp = *((volatile u64*)&S->opp);
+      s_term = *((volatile u32*)&S->term);
+    }
+    __syncthreads();
+    if (!s_go) break;
+    int r;
+    if (s_term) {
+      const int x = __popcll(s_own), y = __popcll(s_opp);
+      r = (x > y) - (x < y);
+    } else {
+      r = playout(s_own, s_opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, &plies);
+    }
+    const u32 bw = __popc(__ballot_sync(kFull, r == 1));
+    const u32 bd = __popc(__ballot_sync(kFull, r == 0));
+    if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
+    __syncthreads();
+    if (tid == 0) {
+      const u32 W = s_w[0] + s_w[1] + s_w[2] + s_w[3];
+      const u32 D = s_d[0] + s_d[1] + s_d[2] + s_d[3];
+      const u32 par = it & 1u;
+      if (W) atomicAdd(&S->wd[par][0], W);
+      if (D) atomicAdd(&S->wd[par][1], D);
+      __threadfence();
+      atomicAdd(&S->arrive, 1u);
+    }
+  }
+  const u32 bp = __reduce_add_sync(kFull, plies);
+  if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
+  if (leader_cta && warp == 0) merge_root(T, 0, unit, it, a.stats, lane);
+}
+
+// ---------------------------------------------------------------------------
+__global__ void ln_table_kernel(double* __restrict__ out, u32 unit, u32 K) {
+  const u32 k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k > K) return;
+  out[k] = k == 0 ? 0.0 : ln_rn((unsigned long long)k * unit);
+}
+
+__global__ void stamp_kernel(u64* t0) { *t0 = globaltimer_ns(); }
+
+// Synthetic positions, one thread per position.
+__global__ void gen_positions_kernel(uint2 key, u32 n, u32 lmin, u32 lmax, DevPosition* out) {
+  const u32 p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= n) return;
+  const u32 span = lmax - lmin + 1u;
+  DevPosition q0;  // attempts are capped (never reached for lmax <= 50): opening
+  q0.black = 0x0000000810000000ULL; q0.white = 0x0000001008000000ULL; q0.to_move = 0; q0.reserved = 0;
+  out[p] = q0;
+  for (u32 attempt = 0; attempt < (1u << 16); ++attempt) {
+    PlayoutRng rng;
+    rng.key = key; rng.c0 = p; rng.c1 = 0xFFFFFFFFu; rng.c2 = attempt; rng.w = 0;
+    rng.buf = make_uint4(0, 0, 0, 0);
+    const u32 L = lmin + __umulhi(rng.next(), span);
+    u64 me = 0x0000000810000000ULL, op = 0x0000001008000000ULL;
+    u32 stm = 0, plies = 0;
+    bool ok = true, passed = false;
+    while (plies < L) {
+      const u64 m = legal_moves(me, op);
+      if (m == 0ULL) {
+        if (passed) { ok = false; break; }
+        passed = true;
+      } else {
+        passed = false;
+        const int sq = pick_square(m, rng.next());
+        const u64 f = flips(sq, me, op);
+        me |= f | (1ULL << sq);
+        op &= ~f;
+        ++plies;
+      }
+      const u64 t = me; me = op; op = t;
+      stm ^= 1u;
+    }
+    if (!ok) continue;
+    if (is_terminal(me, op, legal_moves(me, op))) continue;
+    DevPosition q;
+    q.black = stm == 0u ? me : op;
+    q.white = stm == 0u ? op : me;
+    q.to_move = stm;
+    q.reserved = 0;
+    out[p] = q;
+    return;
+  }
+}
+
+}  // namespace mcts_dev

@@ -1,0 +1,450 @@
+// mcts_api.cu — the C ABI (include/mcts.h) over the sm_100a kernels.
+//
+// Host side only marshals arguments, validates them, owns device scratch
+// (tree pools, ln tables, staging) and launches kernels; every step of the hot
+// path runs on the GPU. There is no CPU fallback: without an sm_100 device the
+// compute calls fail with MCTS_E_NO_DEVICE.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "../../include/mcts.h"
+#include "kernels.cuh"
+
+using namespace mcts_dev;
+
+static_assert(sizeof(mcts_position) == sizeof(DevPosition), "position layout");
+static_assert(sizeof(mcts_wdl) == sizeof(WdlOut), "wdl layout");
+
+struct mcts_handle {
+  int device = 0;
+  mcts_params params{};
+  mcts_position position{};
+  bool has_position = false;
+  cudaStream_t stream = nullptr;  // for the synchronous entry points
+  std::string last_error;
+
+  // playout staging
+  DevPosition* d_leaves = nullptr;
+  size_t leaves_cap = 0;
+  WdlOut* d_wdl = nullptr;
+  size_t wdl_cap = 0;
+  unsigned long long* d_plies = nullptr;
+  void* h_pinned = nullptr;
+  size_t pinned_cap = 0;
+
+  // trees
+  void* pool_mem = nullptr;
+  size_t pool_bytes = 0;
+
+  // ln table
+  double* d_lnT = nullptr;
+  uint32_t lnT_unit = 0;
+  uint32_t lnT_K = 0;
+  size_t lnT_cap = 0;
+
+  // search scratch
+  long long* d_stats = nullptr;
+  unsigned long long* d_t0 = nullptr;
+  int* d_error = nullptr;
+  LeafSync* d_leafsync = nullptr;
+};
+
+namespace {
+
+thread_local std::string g_create_error;
+
+mcts_status fail(mcts_handle* h, mcts_status st, const std::string& msg) {
+  if (h) h->last_error = msg;
+  else g_create_error = msg;
+  return st;
+}
+
+mcts_status cuda_fail(mcts_handle* h, cudaError_t e, const char* where) {
+  std::string msg = std::string(where) + ": " + cudaGetErrorString(e);
+  return fail(h, e == cudaErrorMemoryAllocation ? MCTS_E_OOM : MCTS_E_CUDA, msg);
+}
+
+#define CK(h, call)                                             \
+  do {                                                          \
+    cudaError_t e_ = (call);                                    \
+    if (e_ != cudaSuccess) return cuda_fail((h), e_, #call);    \
+  } while (0)
+
+bool position_ok(const mcts_position& p) {
+  return (p.black & p.white) == 0 && (p.to_move == 0u || p.to_move == 1u);
+}
+
+uint2 key_of(uint64_t seed) { return make_uint2((uint32_t)(seed & 0xFFFFFFFFu), (uint32_t)(seed >> 32)); }
+
+mcts_status ensure(mcts_handle* h, void** ptr, size_t* cap, size_t bytes) {
+  if (*cap >= bytes && *ptr) return MCTS_OK;
+  if (*ptr) { cudaFree(*ptr); *ptr = nullptr; *cap = 0; }
+  size_t want = bytes < 256 ? 256 : bytes;
+  cudaError_t e = cudaMalloc(ptr, want);
+  if (e != cudaSuccess) { *ptr = nullptr; return cuda_fail(h, e, "cudaMalloc"); }
+  *cap = want;
+  return MCTS_OK;
+}
+
+// Device ln table for `unit` with at least K+1 entries (regenerated on demand).
+mcts_status ensure_lnT(mcts_handle* h, uint32_t unit, uint32_t K, cudaStream_t s) {
+  if (h->d_lnT && h->lnT_unit == unit && h->lnT_K >= K) return MCTS_OK;
+  uint32_t Kalloc = K < 1024 ? 1024 : K;
+  size_t bytes = ((size_t)Kalloc + 1) * sizeof(double);
+  if (h->lnT_cap < bytes) {
+    void* p = h->d_lnT;
+    size_t cap = h->lnT_cap;
+    mcts_status st = ensure(h, &p, &cap, bytes);
+    if (st) return st;
+    h->d_lnT = (double*)p;
+    h->lnT_cap = cap;
+  }
+  const uint32_t n = Kalloc + 1;
+  ln_table_kernel<<<(n + 255) / 256, 256, 0, s>>>(h->d_lnT, unit, Kalloc);
+  CK(h, cudaGetLastError());
+  h->lnT_unit = unit;
+  h->lnT_K = Kalloc;
+  return MCTS_OK;
+}
+
+// Carve a TreePool for n_trees * slot_cap slots out of one allocation.
+mcts_status ensure_pool(mcts_handle* h, uint32_t n_trees, uint32_t slot_cap, TreePool* T) {
+  const size_t slots = (size_t)n_trees * slot_cap;
+  const size_t per = 3 * sizeof(u64) + 5 * sizeof(u32);
+  const size_t bytes = slots * per + 8 * 256;
+  if (bytes > (size_t)96 << 30)
+    return fail(h, MCTS_E_OOM, "tree pool would exceed 96 GiB; lower iterations or max_nodes_per_tree");
+  mcts_status st = ensure(h, &h->pool_mem, &h->pool_bytes, bytes);
+  if (st) return st;
+  char* p = (char*)h->pool_mem;
+  auto take = [&](size_t b) { char* q = p; p += (b + 255) & ~(size_t)255; return q; };
+  T->own = (u64*)take(slots * sizeof(u64));
+  T->opp = (u64*)take(slots * sizeof(u64));
+  T->legal = (u64*)take(slots * sizeof(u64));
+  T->k = (u32*)take(slots * sizeof(u32));
+  T->w = (u32*)take(slots * sizeof(u32));
+  T->d = (u32*)take(slots * sizeof(u32));
+  T->first = (u32*)take(slots * sizeof(u32));
+  T->meta = (u32*)take(slots * sizeof(u32));
+  T->slot_cap = slot_cap;
+  return MCTS_OK;
+}
+
+mcts_status check_device(mcts_handle* h) {
+  cudaError_t e = cudaSetDevice(h->device);
+  if (e != cudaSuccess) return fail(h, MCTS_E_NO_DEVICE, std::string("cudaSetDevice: ") + cudaGetErrorString(e));
+  return MCTS_OK;
+}
+
+template <int MAXT, int MINB>
+mcts_status launch_block(mcts_handle* h, uint32_t n_trees, uint32_t threads, const TreePool& T,
+                         const SearchArgs& a, cudaStream_t s) {
+  block_search_kernel<MAXT, MINB><<<n_trees, threads, 0, s>>>(T, a);
+  CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+// The search body shared by mcts_search / mcts_search_async. Writes the
+// MCTS_STATS_LEN sums to d_stats on stream s.
+mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                        uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                        uint32_t tree_id_base, long long* d_stats, cudaStream_t s) {
+  const mcts_position* rp = root ? root : (h->has_position ? &h->position : nullptr);
+  if (!rp) return fail(h, MCTS_E_INVALID_ARGUMENT, "no root position (root == NULL and none given at create)");
+  if (!position_ok(*rp)) return fail(h, MCTS_E_INVALID_POSITION, "root: black & white overlap or bad to_move");
+  const bool by_iter = budget.iterations != 0;
+  const bool by_time = budget.time_ms != 0.0;
+  if (by_iter == by_time) return fail(h, MCTS_E_INVALID_ARGUMENT, "budget: exactly one of iterations / time_ms must be non-zero");
+  if (by_time && !(budget.time_ms > 0.0 && budget.time_ms < 3.6e6))
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "budget.time_ms must be in (0, 3.6e6)");
+  if (n_trees == 0) return fail(h, MCTS_E_INVALID_ARGUMENT, "n_trees == 0");
+  if (!d_stats) return fail(h, MCTS_E_INVALID_ARGUMENT, "d_stats == NULL");
+  const bool leaf = h->params.scheme == MCTS_LEAF;
+  if (leaf) {
+    if (n_trees != 1) return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: n_trees must be 1");
+    if (threads_per_tree == 0 || threads_per_tree % 128 || threads_per_tree > 65536)
+      return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: threads_per_tree must be a multiple of 128 in [128, 65536]");
+  } else {
+    if (threads_per_tree == 0 || threads_per_tree % 32 || threads_per_tree > 1024)
+      return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_BLOCK: threads_per_tree must be a multiple of 32 in [32, 1024] (PAPER.md L310-L311)");
+  }
+  const uint64_t unit = threads_per_tree;
+  const uint64_t kmax_counts = 0xFFFFFFFFull / unit;  // node counters are u32
+  uint64_t max_it;
+  uint32_t slot_cap;
+  if (by_iter) {
+    if (budget.iterations > kmax_counts || budget.iterations > (1u << 24))
+      return fail(h, MCTS_E_INVALID_ARGUMENT, "iterations * threads_per_tree must be < 2^32 and iterations <= 2^24");
+    max_it = budget.iterations;
+    // Each expanded interior node reserves <= 60 child slots; at most one node
+    // is expanded per iteration, so the pool never fills (oracle capacity =
+    // iterations + 1 is never reached either).
+    const uint64_t need = 1 + max_it * 60;
+    slot_cap = (uint32_t)(need > 0xFFFFFFF0ull ? 0xFFFFFFF0ull : need);
+  } else {
+    max_it = kmax_counts < (1u << 20) ? kmax_counts : (1u << 20);
+    slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree : 65536u;
+    if (slot_cap < 64) slot_cap = 64;
+  }
+
+  mcts_status st = check_device(h);
+  if (st) return st;
+  TreePool T;
+  st = ensure_pool(h, n_trees, slot_cap, &T);
+  if (st) return st;
+  st = ensure_lnT(h, (uint32_t)unit, (uint32_t)max_it, s);
+  if (st) return st;
+  CK(h, cudaMemsetAsync(d_stats, 0, MCTS_STATS_LEN * sizeof(long long), s));
+  CK(h, cudaMemsetAsync(h->d_error, 0, sizeof(int), s));
+
+  SearchArgs a;
+  memcpy(&a.root, rp, sizeof(DevPosition));
+  a.key = key_of(seed);
+  a.C = h->params.c_uct;
+  a.lnT = h->d_lnT;
+  a.stats = d_stats;
+  a.t0 = h->d_t0;
+  a.budget_ns = by_time ? (u64)llround(budget.time_ms * 1e6) : 0ULL;
+  if (by_time && a.budget_ns == 0) a.budget_ns = 1;
+  a.max_iterations = (u32)max_it;
+  a.tree_id_base = tree_id_base;
+  a.unit = (u32)unit;
+  a.error = h->d_error;
+  if (by_time) {
+    stamp_kernel<<<1, 1, 0, s>>>(h->d_t0);
+    CK(h, cudaGetLastError());
+  }
+
+  if (!leaf) {
+    if (threads_per_tree <= 128) return launch_block<128, 8>(h, n_trees, threads_per_tree, T, a, s);
+    if (threads_per_tree <= 256) return launch_block<256, 4>(h, n_trees, threads_per_tree, T, a, s);
+    if (threads_per_tree <= 512) return launch_block<512, 2>(h, n_trees, threads_per_tree, T, a, s);
+    return launch_block<1024, 1>(h, n_trees, threads_per_tree, T, a, s);
+  }
+  // leaf parallelism: one cooperative grid of unit/128 co-resident CTAs
+  const uint32_t G = threads_per_tree / 128;
+  int per_sm = 0, n_sm = 0;
+  CK(h, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, leaf_search_kernel, 128, 0));
+  CK(h, cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, h->device));
+  if ((long long)per_sm * n_sm < (long long)G)
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: batch does not fit co-resident on the device");
+  CK(h, cudaMemsetAsync(h->d_leafsync, 0, sizeof(LeafSync), s));
+  LeafSync* S = h->d_leafsync;
+  void* args[] = {(void*)&T, (void*)&a, (void*)&S};
+  CK(h, cudaLaunchCooperativeKernel((const void*)leaf_search_kernel, dim3(G), dim3(128), args, 0, s));
+  return MCTS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* mcts_version(void) { return "mcts-b200 0.1 (sm_100a)"; }
+
+const char* mcts_status_string(mcts_status st) {
+  switch (st) {
+    case MCTS_OK: return "MCTS_OK";
+    case MCTS_E_INVALID_ARGUMENT: return "MCTS_E_INVALID_ARGUMENT";
+    case MCTS_E_INVALID_POSITION: return "MCTS_E_INVALID_POSITION";
+    case MCTS_E_CUDA: return "MCTS_E_CUDA";
+    case MCTS_E_OOM: return "MCTS_E_OOM";
+    case MCTS_E_NO_DEVICE: return "MCTS_E_NO_DEVICE";
+    default: return "MCTS_E_UNKNOWN";
+  }
+}
+
+const char* mcts_last_error(const mcts_handle* h) {
+  return h ? h->last_error.c_str() : g_create_error.c_str();
+}
+
+mcts_status mcts_create(const mcts_position* position, const mcts_params* params, mcts_handle** out) {
+  if (!out || !params) return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "out / params is NULL");
+  *out = nullptr;
+  if (params->scheme != MCTS_BLOCK && params->scheme != MCTS_LEAF)
+    return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->scheme must be MCTS_BLOCK or MCTS_LEAF");
+  if (!std::isfinite(params->c_uct) || params->c_uct < 0.0)
+    return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->c_uct must be finite and >= 0");
+  if (position && !position_ok(*position))
+    return fail(nullptr, MCTS_E_INVALID_POSITION, "position: black & white overlap or bad to_move");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0)
+    return fail(nullptr, MCTS_E_NO_DEVICE, std::string("no CUDA device: ") + cudaGetErrorString(e));
+  if (params->device < 0 || params->device >= ndev)
+    return fail(nullptr, MCTS_E_NO_DEVICE, "params->device out of range");
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, params->device);
+  if (e != cudaSuccess) return fail(nullptr, MCTS_E_NO_DEVICE, cudaGetErrorString(e));
+  if (prop.major != 10)
+    return fail(nullptr, MCTS_E_NO_DEVICE, "device is not compute capability 10.x (built for sm_100a only)");
+  mcts_handle* h = new mcts_handle();
+  h->device = params->device;
+  h->params = *params;
+  if (position) { h->position = *position; h->has_position = true; }
+  e = cudaSetDevice(h->device);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_stats, MCTS_STATS_LEN * sizeof(long long));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_t0, sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_error, sizeof(int));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_plies, sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_leafsync, sizeof(LeafSync));
+  if (e != cudaSuccess) {
+    g_create_error = std::string("mcts_create: ") + cudaGetErrorString(e);
+    mcts_destroy(h);
+    return e == cudaErrorMemoryAllocation ? MCTS_E_OOM : MCTS_E_CUDA;
+  }
+  *out = h;
+  return MCTS_OK;
+}
+
+void mcts_destroy(mcts_handle* h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  cudaFree(h->d_leaves);
+  cudaFree(h->d_wdl);
+  cudaFree(h->d_plies);
+  cudaFree(h->pool_mem);
+  cudaFree(h->d_lnT);
+  cudaFree(h->d_stats);
+  cudaFree(h->d_t0);
+  cudaFree(h->d_error);
+  cudaFree(h->d_leafsync);
+  if (h->h_pinned) cudaFreeHost(h->h_pinned);
+  if (h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+}
+
+mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
+                                uint32_t n_per_leaf, uint64_t seed, uint32_t leaf_id_base,
+                                mcts_wdl* d_out, uint64_t* d_plies, void* stream) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (n_leaves && (!d_leaves || !d_out)) return fail(h, MCTS_E_INVALID_ARGUMENT, "NULL leaves / out");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n_leaves == 0) return MCTS_OK;
+  CK(h, cudaMemsetAsync(d_out, 0, (size_t)n_leaves * sizeof(mcts_wdl), s));
+  const uint64_t total = (uint64_t)n_leaves * n_per_leaf;
+  if (total == 0) return MCTS_OK;
+  const uint64_t blocks = (total + kPlayoutThreads - 1) / kPlayoutThreads;
+  if (blocks > 0x7FFFFFFFull) return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large");
+  playouts_kernel<<<(unsigned)blocks, kPlayoutThreads, 0, s>>>(
+      (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), leaf_id_base, (WdlOut*)d_out,
+      (unsigned long long*)d_plies);
+  CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
+                          uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts, uint64_t* out_plies) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (out_plies) *out_plies = 0;
+  if (n_leaves == 0) return MCTS_OK;
+  if (!leaf_batch || !out_counts) return fail(h, MCTS_E_INVALID_ARGUMENT, "NULL leaf_batch / out_counts");
+  for (uint32_t i = 0; i < n_leaves; ++i)
+    if (!position_ok(leaf_batch[i]))
+      return fail(h, MCTS_E_INVALID_POSITION, "leaf " + std::to_string(i) + ": black & white overlap or bad to_move");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  void* p = h->d_leaves;
+  st = ensure(h, &p, &h->leaves_cap, (size_t)n_leaves * sizeof(DevPosition));
+  if (st) return st;
+  h->d_leaves = (DevPosition*)p;
+  p = h->d_wdl;
+  st = ensure(h, &p, &h->wdl_cap, (size_t)n_leaves * sizeof(WdlOut));
+  if (st) return st;
+  h->d_wdl = (WdlOut*)p;
+  cudaStream_t s = h->stream;
+  CK(h, cudaMemsetAsync(h->d_plies, 0, sizeof(unsigned long long), s));
+  CK(h, cudaMemcpyAsync(h->d_leaves, leaf_batch, (size_t)n_leaves * sizeof(DevPosition), cudaMemcpyHostToDevice, s));
+  st = mcts_playouts_async(h, (const mcts_position*)h->d_leaves, n_leaves, n_per_leaf, seed, 0,
+                           (mcts_wdl*)h->d_wdl, (uint64_t*)h->d_plies, s);
+  if (st) return st;
+  CK(h, cudaMemcpyAsync(out_counts, h->d_wdl, (size_t)n_leaves * sizeof(WdlOut), cudaMemcpyDeviceToHost, s));
+  unsigned long long plies = 0;
+  CK(h, cudaMemcpyAsync(&plies, h->d_plies, sizeof(plies), cudaMemcpyDeviceToHost, s));
+  CK(h, cudaStreamSynchronize(s));
+  if (out_plies) *out_plies = plies;
+  return MCTS_OK;
+}
+
+mcts_status mcts_search_async(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                              uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                              uint32_t tree_id_base, int64_t* d_stats, void* stream) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  return search_impl(h, root, budget, n_trees, threads_per_tree, seed, tree_id_base,
+                     (long long*)d_stats, (cudaStream_t)stream);
+}
+
+int32_t mcts_best_move(const int64_t* stats) {
+  if (!stats) return -1;
+  int32_t best = -1;
+  int64_t bv = 0;
+  for (int mv = 0; mv < 65; ++mv)
+    if (stats[mv] > bv) { bv = stats[mv]; best = mv; }
+  return best;
+}
+
+mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                        uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                        mcts_root_stats* out) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (!out) return fail(h, MCTS_E_INVALID_ARGUMENT, "out == NULL");
+  mcts_status st = search_impl(h, root, budget, n_trees, threads_per_tree, seed, 0, h->d_stats, h->stream);
+  if (st) return st;
+  long long hs[MCTS_STATS_LEN];
+  CK(h, cudaMemcpyAsync(hs, h->d_stats, sizeof(hs), cudaMemcpyDeviceToHost, h->stream));
+  int herr = 0;
+  CK(h, cudaMemcpyAsync(&herr, h->d_error, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CK(h, cudaStreamSynchronize(h->stream));
+  if (herr) return fail(h, MCTS_E_CUDA, "leaf search watchdog fired (grid barrier did not complete)");
+  for (int i = 0; i < 65; ++i) {
+    out->visits[i] = (uint64_t)hs[i];
+    out->wins[i] = (uint64_t)hs[65 + i];
+    out->draws[i] = (uint64_t)hs[130 + i];
+  }
+  out->root_visits = (uint64_t)hs[195];
+  out->iterations_done = (uint64_t)hs[196];
+  out->plies = (uint64_t)hs[197];
+  out->best_move = mcts_best_move((const int64_t*)hs);
+  out->reserved = 0;
+  return MCTS_OK;
+}
+
+mcts_status mcts_gen_positions_async(mcts_handle* h, uint64_t seed, uint32_t n, uint32_t lmin,
+                                     uint32_t lmax, mcts_position* d_out, void* stream) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (lmin > lmax || lmax > 50) return fail(h, MCTS_E_INVALID_ARGUMENT, "need lmin <= lmax <= 50");
+  if (n && !d_out) return fail(h, MCTS_E_INVALID_ARGUMENT, "d_out == NULL");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  if (n == 0) return MCTS_OK;
+  gen_positions_kernel<<<(n + 127) / 128, 128, 0, (cudaStream_t)stream>>>(key_of(seed), n, lmin, lmax,
+                                                                         (DevPosition*)d_out);
+  CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+mcts_status mcts_ln_table(mcts_handle* h, uint32_t unit, uint32_t K, double* out) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (!out || unit == 0) return fail(h, MCTS_E_INVALID_ARGUMENT, "out == NULL or unit == 0");
+  if ((uint64_t)K * unit >= (1ull << 53)) return fail(h, MCTS_E_INVALID_ARGUMENT, "K * unit must be < 2^53");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  double* d = nullptr;
+  CK(h, cudaMalloc(&d, ((size_t)K + 1) * sizeof(double)));
+  ln_table_kernel<<<(K + 1 + 255) / 256, 256, 0, h->stream>>>(d, unit, K);
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(out, d, ((size_t)K + 1) * sizeof(double), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  cudaFree(d);
+  if (e != cudaSuccess) return cuda_fail(h, e, "mcts_ln_table");
+  return MCTS_OK;
+}
+
+}  // extern "C"

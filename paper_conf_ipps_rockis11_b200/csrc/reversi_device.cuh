@@ -1,0 +1,171 @@
+// reversi_device.cuh — device game core for the playout hot loop (sm_100a).
+//
+// Bitboard 8x8 Reversi: square s = 8*row + col, bit s of a uint64 (DESIGN.md
+// §3 R7). Everything here is plain integer/bit work on the ALU and FMA pipes:
+// shift-mask move generation, a branch-free popc binary search for the random
+// pick, shift-mask flips and a counter-based Philox4x32-10. See DESIGN.md §6
+// for the per-ply instruction budget these functions set.
+//
+// PAPER.md L149-L151 (§II): "A simulation is defined as a series of random
+// moves which are performed until the end of a game is reached (until neither
+// of the players can move)."
+#pragma once
+#include <cstdint>
+
+namespace mcts_dev {
+
+typedef unsigned long long u64;
+typedef uint32_t u32;
+
+// Propagator mask for directions with a column component: an opponent disc on
+// file a or h can never be bracketed along a horizontal or diagonal line.
+constexpr u64 kInner = 0x7E7E7E7E7E7E7E7EULL;
+
+template <int S>
+__device__ __forceinline__ u64 sh(u64 x) {
+  if constexpr (S > 0) return x << S;
+  else return x >> (-S);
+}
+
+// Moves of P against O along direction S: a run of >= 1 propagator discs M
+// attached to P, continued by one more step (the landing square). 6 fill steps
+// cover the longest possible run (6 discs between two squares of a line).
+template <int S>
+__device__ __forceinline__ u64 dir_moves(u64 P, u64 M) {
+  u64 t = M & sh<S>(P);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  return sh<S>(t);
+}
+
+// Legal-move mask of the side owning P (opponent O).
+__device__ __forceinline__ u64 legal_moves(u64 P, u64 O) {
+  const u64 M = O & kInner;
+  u64 m = dir_moves<1>(P, M) | dir_moves<-1>(P, M);
+  m |= dir_moves<8>(P, O) | dir_moves<-8>(P, O);
+  m |= dir_moves<7>(P, M) | dir_moves<-7>(P, M);
+  m |= dir_moves<9>(P, M) | dir_moves<-9>(P, M);
+  return m & ~(P | O);
+}
+
+// Discs flipped along direction S when P plays the square x (a single bit):
+// the contiguous propagator run starting next to x, kept only if the square
+// after it holds a P disc.
+template <int S>
+__device__ __forceinline__ u64 dir_flips(u64 x, u64 P, u64 M) {
+  u64 t = M & sh<S>(x);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  t |= M & sh<S>(t);
+  return (sh<S>(t) & P) ? t : 0ULL;
+}
+
+__device__ __forceinline__ u64 flips(int sq, u64 P, u64 O) {
+  const u64 x = 1ULL << sq;
+  const u64 M = O & kInner;
+  u64 f = dir_flips<1>(x, P, M) | dir_flips<-1>(x, P, M);
+  f |= dir_flips<8>(x, P, O) | dir_flips<-8>(x, P, O);
+  f |= dir_flips<7>(x, P, M) | dir_flips<-7>(x, P, M);
+  f |= dir_flips<9>(x, P, M) | dir_flips<-9>(x, P, M);
+  return f;
+}
+
+// Index (0..63) of the k-th set bit (k = 0: lowest) of m; k < popc(m).
+// Branch-free binary search on population counts.
+__device__ __forceinline__ int kth_set_bit(u64 m, u32 k) {
+  u32 lo = (u32)m, hi = (u32)(m >> 32);
+  u32 c = __popc(lo);
+  bool up = k >= c;
+  u32 x = up ? hi : lo;
+  k -= up ? c : 0u;
+  int base = up ? 32 : 0;
+  c = __popc(x & 0xFFFFu); up = k >= c; x = up ? (x >> 16) : x; k -= up ? c : 0u; base += up ? 16 : 0;
+  c = __popc(x & 0xFFu);   up = k >= c; x = up ? (x >> 8) : x;  k -= up ? c : 0u; base += up ? 8 : 0;
+  c = __popc(x & 0xFu);    up = k >= c; x = up ? (x >> 4) : x;  k -= up ? c : 0u; base += up ? 4 : 0;
+  c = __popc(x & 0x3u);    up = k >= c; x = up ? (x >> 2) : x;  k -= up ? c : 0u; base += up ? 2 : 0;
+  c = x & 1u;              up = k >= c;                                           base += up ? 1 : 0;
+  return base;
+}
+
+// Uniform pick (R4): k = floor(r * c / 2^32), then the k-th legal
+// square in ascending order.
+__device__ __forceinline__ int pick_square(u64 moves, u32 r) {
+  u32 c = (u32)__popcll(moves);
+  return kth_set_bit(moves, __umulhi(r, c));
+}
+
+// Philox4x32-10 (Salmon et al. SC'11; cuRAND/Random123 round and constants).
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+  for (int i = 0; i < 10; ++i) {
+    const u32 hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const u32 hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+    k.x += 0x9E3779B9u;
+    k.y += 0xBB67AE85u;
+  }
+  return c;
+}
+
+// Stream of RNG words for one playout (R5): word w is output[w % 4]
+// of Philox(counter = (c0, c1, c2, w / 4), key = seed).
+struct PlayoutRng {
+  uint2 key;
+  u32 c0, c1, c2;
+  u32 w;
+  uint4 buf;
+  __device__ __forceinline__ u32 next() {
+    const u32 lane = w & 3u;
+    if (lane == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
+    ++w;
+    u32 r = buf.x;
+    r = lane == 1u ? buf.y : r;
+    r = lane == 2u ? buf.z : r;
+    r = lane == 3u ? buf.w : r;
+    return r;
+  }
+};
+
+// One random playout from (me to move, op). Returns +1 / 0 / -1 for the side
+// to move at the start (R3), adds the non-pass plies to *plies.
+// A pass consumes no RNG word; two consecutive passes end the game.
+__device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1, u32 c2,
+                                       u32* plies) {
+  PlayoutRng rng;
+  rng.key = key; rng.c0 = c0; rng.c1 = c1; rng.c2 = c2; rng.w = 0;
+  rng.buf = make_uint4(0, 0, 0, 0);
+  bool start = true;   // does `me` belong to the player who was to move at the start?
+  bool passed = false;
+  u32 n = 0;
+  for (;;) {
+    const u64 moves = legal_moves(me, op);
+    if (moves == 0ULL) {
+      if (passed) break;  // neither player can move
+      passed = true;
+    } else {
+      passed = false;
+      const int sq = pick_square(moves, rng.next());
+      const u64 f = flips(sq, me, op);
+      me |= f | (1ULL << sq);
+      op &= ~f;
+      ++n;
+    }
+    const u64 t = me; me = op; op = t;
+    start = !start;
+  }
+  *plies += n;
+  const int a = __popcll(start ? me : op), b = __popcll(start ? op : me);
+  return (a > b) - (a < b);
+}
+
+// Terminal test: neither side has a move.
+__device__ __forceinline__ bool is_terminal(u64 P, u64 O, u64 legalP) {
+  return legalP == 0ULL && legal_moves(O, P) == 0ULL;
+}
+
+}  // namespace mcts_dev

@@ -1,0 +1,183 @@
+// tree_device.cuh — device-resident UCT tree (§II-A).
+//
+// One pool of node slots per tree in HBM, structure-of-arrays so the 32 lanes
+// of the selecting warp read 32 sibling statistics with one coalesced load per
+// field. A node's children occupy a contiguous block of `limit` slots that is
+// reserved the first time the node is expanded; children are created one per
+// iteration (L181 "I add one node per iteration") in ascending move order, so
+// child i of a node is its i-th legal move (or the pass child, move 64).
+//
+// Visit counts are stored in iterations (k); n = k * unit. This is exact: every
+// visit of a node adds `unit` playouts (L186-L195), and it indexes the ln table
+// lnT[k] = RN(ln(k * unit)) directly (R9).
+#pragma once
+#include <cstdint>
+#include "reversi_device.cuh"
+
+namespace mcts_dev {
+
+constexpr u32 kNoChild = 0xFFFFFFFFu;
+constexpr int kMaxPath = 160;  // > 60 moves + passes + root
+constexpr unsigned kFull = 0xFFFFFFFFu;
+
+struct TreePool {
+  u64* own;    // discs of the side to move at the node
+  u64* opp;    // discs of the other side
+  u64* legal;  // legal moves of the side to move
+  u32* k;      // iterations through the node (n = k * unit)
+  u32* w;      // playouts won by mover(node) = the side that moved into it
+  u32* d;      // drawn playouts
+  u32* first;  // first child slot (tree-relative) or kNoChild
+  u32* meta;   // nchild | limit << 8 | move << 16 | terminal << 24
+  u32 slot_cap;
+};
+
+__device__ __forceinline__ u32 meta_nchild(u32 m) { return m & 0xFFu; }
+__device__ __forceinline__ u32 meta_limit(u32 m) { return (m >> 8) & 0xFFu; }
+__device__ __forceinline__ u32 meta_move(u32 m) { return (m >> 16) & 0xFFu; }
+__device__ __forceinline__ bool meta_term(u32 m) { return (m >> 24) != 0u; }
+
+__device__ __forceinline__ void init_node(const TreePool& T, size_t s, u64 own, u64 opp, u32 move) {
+  const u64 lg = legal_moves(own, opp);
+  const bool term = is_terminal(own, opp, lg);
+  const u32 limit = term ? 0u : (lg ? (u32)__popcll(lg) : 1u);
+  T.own[s] = own;
+  T.opp[s] = opp;
+  T.legal[s] = lg;
+  T.k[s] = 0;
+  T.w[s] = 0;
+  T.d[s] = 0;
+  T.first[s] = kNoChild;
+  T.meta[s] = (limit << 8) | (move << 16) | ((term ? 1u : 0u) << 24);
+}
+
+// u = w/n + C*sqrt(lnT[k_parent]/n): five IEEE round-to-nearest operations in
+// this order, no contraction (R1) — bit-identical to the oracle.
+__device__ __forceinline__ double ucb_value(u32 w, u32 k, u32 unit, double ln_parent, double C) {
+  const double n = (double)((unsigned long long)k * unit);
+  const double exploit = __ddiv_rn((double)w, n);
+  const double explore = __dmul_rn(C, __dsqrt_rn(__ddiv_rn(ln_parent, n)));
+  return __dadd_rn(exploit, explore);
+}
+
+struct LeafInfo {
+  u64 own, opp;
+  u32 term;
+  int depth;
+};
+
+// Selection + expansion of one iteration, executed by one full warp.
+// path (shared) receives the node slots root..leaf; *slot_used (shared) is the
+// tree's slot allocator. Returns the leaf (same value in every lane).
+__device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base, u32* path,
+                                                  u32* slot_used, const double* __restrict__ lnT,
+                                                  u32 unit, double C, int lane) {
+  u32 v = 0;
+  int depth = 0;
+  if (lane == 0) path[0] = 0;
+  u32 meta = T.meta[base];
+  // Selection (L157-L178): descend while the node is non-terminal and fully expanded.
+  while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta)) {
+    const u32 nch = meta_nchild(meta);
+    const u32 first = T.first[base + v];
+    const double lnp = lnT[T.k[base + v]];
+    double best_u = -__longlong_as_double(0x7FF0000000000000LL);  // -inf
+    u32 best_i = kNoChild;
+    for (u32 i = (u32)lane; i < nch; i += 32u) {
+      const size_t c = base + first + i;
+      const double u = ucb_value(T.w[c], T.k[c], unit, lnp, C);
+      if (u > best_u) { best_u = u; best_i = i; }
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      const double ou = __shfl_xor_sync(kFull, best_u, off);
+      const u32 oi = __shfl_xor_sync(kFull, best_i, off);
+      if (ou > best_u || (ou == best_u && oi < best_i)) { best_u = ou; best_i = oi; }
+    }
+    v = first + best_i;
+    ++depth;
+    if (lane == 0) path[depth] = v;
+    meta = T.meta[base + v];
+  }
+  // Expansion (L179-L182): the lowest-index untried move, or the pass child.
+  LeafInfo L;
+  if (!meta_term(meta)) {
+    u32 c = kNoChild;
+    if (lane == 0) {
+      const u32 nch = meta_nchild(meta), limit = meta_limit(meta);
+      u32 first = T.first[base + v];
+      if (nch == 0u) {
+        if (*slot_used + limit <= T.slot_cap) {
+          first = *slot_used;
+          *slot_used += limit;
+          T.first[base + v] = first;
+        } else {
+          first = kNoChild;  // pool full (time mode): simulate from v itself
+        }
+      }
+      if (first != kNoChild) {
+        const u64 own = T.own[base + v], opp = T.opp[base + v], lg = T.legal[base + v];
+        c = first + nch;
+        if (lg == 0ULL) {
+          init_node(T, base + c, opp, own, 64u);  // pass: same discs, turn swaps
+        } else {
+          const int sq = kth_set_bit(lg, nch);
+          const u64 f = flips(sq, own, opp);
+          init_node(T, base + c, opp & ~f, own | f | (1ULL << sq), (u32)sq);
+        }
+        T.meta[base + v] = meta + 1u;  // ++nchild
+        path[depth + 1] = c;
+      }
+    }
+    c = __shfl_sync(kFull, c, 0);
+    __syncwarp();
+    if (c != kNoChild) {
+      v = c;
+      ++depth;
+    }
+  }
+  L.own = T.own[base + v];
+  L.opp = T.opp[base + v];
+  L.term = meta_term(T.meta[base + v]) ? 1u : 0u;
+  L.depth = depth;
+  return L;
+}
+
+// Backpropagation (L196-L199) by one warp, lanes over path positions (distinct
+// nodes). W/D/Lo are the leaf batch's wins/draws/losses for the leaf's side to
+// move; the leaf's mover collects Lo, its parent W, alternating to the root.
+__device__ __forceinline__ void backprop(const TreePool& T, size_t base, const u32* path, int depth,
+                                         u32 W, u32 D, u32 Lo, int lane) {
+  for (int p = lane; p <= depth; p += 32) {
+    const size_t s = base + path[p];
+    const int lvl = depth - p;
+    T.k[s] += 1u;
+    T.w[s] += (lvl & 1) ? W : Lo;
+    T.d[s] += D;
+  }
+  __syncwarp();
+}
+
+// Fused root merge (a10): add this tree's root-child statistics into the int64
+// stats vector (see MCTS_STATS_LEN in include/mcts.h). Integer atomics are
+// order-independent, so the sum is deterministic.
+__device__ __forceinline__ void merge_root(const TreePool& T, size_t base, u32 unit, u32 iterations,
+                                           long long* stats, int lane) {
+  const u32 meta = T.meta[base];
+  const u32 nch = meta_nchild(meta);
+  const u32 first = T.first[base];
+  unsigned long long* st = reinterpret_cast<unsigned long long*>(stats);
+  for (u32 i = (u32)lane; i < nch; i += 32u) {
+    const size_t c = base + first + i;
+    const u32 mv = meta_move(T.meta[c]);
+    atomicAdd(st + mv, (unsigned long long)T.k[c] * unit);
+    atomicAdd(st + 65 + mv, (unsigned long long)T.w[c]);
+    atomicAdd(st + 130 + mv, (unsigned long long)T.d[c]);
+  }
+  if (lane == 0) {
+    atomicAdd(st + 195, (unsigned long long)T.k[base] * unit);
+    atomicAdd(st + 196, (unsigned long long)iterations);
+  }
+}
+
+}  // namespace mcts_dev

@@ -1,0 +1,262 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, element by element.
+
+Bar: bit-exact for everything — W/D/L counts, ply counts,
+generated positions, the ln table, and the full UCT root statistics and best
+move in iteration mode (the UCB arithmetic is correctly rounded IEEE double on
+both sides). Time mode is checked by invariants only (parity unpinned).
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_ipps_rockis11_b200 as pkg
+from paper_conf_ipps_rockis11_b200 import device as dev
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def mcts():
+    m = pkg.Mcts(c_uct=1.0, scheme="block", device=0)
+    yield m
+    m.close()
+
+
+@pytest.fixture(scope="module")
+def mcts_leaf():
+    m = pkg.Mcts(c_uct=1.0, scheme="leaf", device=0)
+    yield m
+    m.close()
+
+
+# ---------------------------------------------------------------- ln table
+@pytest.mark.parametrize("unit,K", [(1, 200000), (32, 50000), (64, 50000), (128, 50000),
+                                    (16384, 20000), (1000, 1000)])
+def test_ln_table_bitwise(mcts, orc, unit, K):
+    got = mcts.ln_table(unit, K)
+    want = orc.ln_table(unit, K)
+    assert got.view(np.uint64).tolist() == want.view(np.uint64).tolist()
+
+
+def test_ln_regression_and_large(mcts, orc):
+    assert mcts.ln_table(9170, 1)[1] == float.fromhex("0x1.23f54a1c504c1p+3")
+    big = mcts.ln_table(1 << 20, 4096)
+    assert (big == orc.ln_table(1 << 20, 4096)).all()
+
+
+# ---------------------------------------------------------------- generator
+@pytest.mark.parametrize("seed,n,lmin,lmax", [(2, 4096, 20, 40), (1, 4096, 0, 8), (7, 1000, 40, 50),
+                                              (3, 5, 0, 0), (4, 333, 10, 10)])
+def test_gen_positions(mcts, orc, seed, n, lmin, lmax):
+    got = dev.tensor_to_positions(dev.gen_positions(mcts, seed, n, lmin, lmax))
+    want = orc.gen_positions(seed, n, lmin, lmax)
+    assert (got["black"] == want["black"]).all()
+    assert (got["white"] == want["white"]).all()
+    assert (got["to_move"] == want["to_move"]).all()
+
+
+# ---------------------------------------------------------------- playouts
+@pytest.mark.parametrize("seed,n,per,lmin,lmax", [
+    (2, 256, 64, 20, 40),     # several tiles of the c1 recipe
+    (5, 77, 37, 20, 40),      # ragged: n_per_leaf not a multiple of 32
+    (6, 300, 1, 0, 50),       # one playout per leaf, warps span 32 leaves
+    (1, 64, 96, 0, 8),        # opening phase (~60-ply playouts)
+    (9, 50, 33, 40, 50),      # late game, frequent passes
+])
+def test_playouts_bit_exact(mcts, orc, seed, n, per, lmin, lmax):
+    leaves = orc.gen_positions(seed, n, lmin, lmax)
+    wdl, plies = mcts.playouts(leaves, per, seed=seed * 1000 + 7)
+    owdl, oplies = orc.playouts(leaves, per, seed=seed * 1000 + 7)
+    assert (wdl == owdl).all()
+    assert plies == oplies
+
+
+def test_playouts_edge_cases(mcts, orc):
+    full_black = (1 << 40) - 1
+    full_white = ((1 << 64) - 1) & ~full_black
+    leaves = np.concatenate([
+        orc.position(full_black, full_white, 0),     # terminal, win
+        orc.position(full_black, full_white, 1),     # terminal, loss
+        orc.position((1 << 32) - 1, ((1 << 64) - 1) & ~((1 << 32) - 1), 0),  # terminal draw
+        orc.position(0b11, 0b100, 1),                # must pass first
+        orc.opening(),
+    ])
+    wdl, plies = mcts.playouts(leaves, 45, seed=11)
+    owdl, oplies = orc.playouts(leaves, 45, seed=11)
+    assert (wdl == owdl).all() and plies == oplies
+    assert wdl[0].tolist() == [45, 0, 0] and wdl[1].tolist() == [0, 0, 45] and wdl[2].tolist() == [0, 45, 0]
+    # n_per_leaf == 0 and n_leaves == 0
+    z, zp = mcts.playouts(leaves, 0, seed=1)
+    assert (z == 0).all() and zp == 0
+    e, ep = mcts.playouts(leaves[:0], 10, seed=1)
+    assert e.shape == (0, 3) and ep == 0
+
+
+def test_playouts_invalid_position(mcts, orc):
+    bad = orc.position(1, 1, 0)
+    with pytest.raises(pkg.MctsError) as ei:
+        mcts.playouts(bad, 4, seed=1)
+    assert ei.value.status == -2
+
+
+def test_playouts_full_size_sampled(mcts, orc):
+    """BASELINE configs[1] at full size (4096 x 256) in the bench's launch
+    configuration (async, device buffers); oracle on sampled leaves."""
+    n, per, seed = 4096, 256, 2
+    d_leaves = dev.gen_positions(mcts, seed, n, 20, 40)
+    d_out = dev.empty_wdl(n)
+    d_plies = torch.zeros(1, dtype=torch.int64, device="cuda")
+    mcts.playouts_async(d_leaves.data_ptr(), n, per, seed, 0, d_out.data_ptr(), d_plies.data_ptr(),
+                        torch.cuda.current_stream())
+    torch.cuda.synchronize()
+    wdl = d_out.cpu().numpy()
+    assert (wdl.sum(axis=1) == per).all()
+    leaves = orc.gen_positions(seed, n, 20, 40)
+    rng = np.random.default_rng(0)
+    idx = np.sort(rng.choice(n, 24, replace=False))
+    idx = np.concatenate([[0, n - 1], idx])
+    for i in idx:
+        owdl, _ = orc.playouts(leaves[i:i + 1], per, seed=seed, leaf_id_base=int(i))
+        assert wdl[i].tolist() == owdl[0].tolist(), i
+    # plies: property at any size — between 1 and the empties per playout
+    empties = 64 - np.array([bin(int(b) | int(w)).count("1") for b, w in zip(leaves["black"], leaves["white"])])
+    assert int(d_plies.item()) <= int(empties.sum()) * per
+    assert int(d_plies.item()) >= int(empties.sum()) * per * 0.9
+
+
+def test_playouts_leaf_range_sharding(mcts, orc):
+    """Splitting a batch by leaf range with leaf_id_base reproduces one call."""
+    n, per, seed = 500, 32, 3
+    d_leaves = dev.gen_positions(mcts, seed, n, 20, 40)
+    whole = dev.empty_wdl(n)
+    mcts.playouts_async(d_leaves.data_ptr(), n, per, seed, 0, whole.data_ptr(), 0, None)
+    parts = dev.empty_wdl(n)
+    from paper_conf_ipps_rockis11_b200.distributed import leaf_range
+    for r in range(3):
+        a, b = leaf_range(r, 3, n)
+        mcts.playouts_async(d_leaves[a:].data_ptr(), b - a, per, seed, a, parts[a:].data_ptr(), 0, None)
+    torch.cuda.synchronize()
+    assert torch.equal(whole, parts)
+
+
+# ---------------------------------------------------------------- search
+def _cmp_search(res, ostats, obest):
+    assert res["stats"][:197].tolist() == ostats[:197].tolist()
+    assert res["best_move"] == obest
+
+
+def test_search_config0_bit_exact(mcts, orc):
+    """BASELINE configs[0]: opening, 1 tree x 64 threads x 100 iterations, seed 1."""
+    res = mcts.search(pkg.opening(), iterations=100, n_trees=1, threads_per_tree=64, seed=1)
+    ostats, obest, oplies = orc.uct_search(orc.opening(), 1, 64, 100, 1)
+    _cmp_search(res, ostats, obest)
+    assert res["plies"] == oplies
+    assert res["root_visits"] == 6400 and res["iterations"] == 100
+
+
+@pytest.mark.parametrize("n_trees,threads,iters,seed,C,lmin,lmax", [
+    (8, 32, 300, 4, 1.0, 20, 40),
+    (3, 256, 40, 5, 0.5, 10, 30),
+    (5, 96, 60, 6, 2.0, 30, 50),
+    (2, 1024, 12, 7, 1.0, 0, 8),
+    (4, 64, 200, 8, 0.0, 20, 40),
+])
+def test_search_block_bit_exact(orc, n_trees, threads, iters, seed, C, lmin, lmax):
+    m = pkg.Mcts(c_uct=C, scheme="block", device=0)
+    root = orc.gen_positions(seed, 1, lmin, lmax)
+    res = m.search(root, iterations=iters, n_trees=n_trees, threads_per_tree=threads, seed=seed)
+    ostats, obest, oplies = orc.uct_search(root, n_trees, threads, iters, seed, C=C)
+    _cmp_search(res, ostats, obest)
+    assert res["plies"] == oplies
+    m.close()
+
+
+def test_search_config2_iteration_mode(mcts, orc):
+    """BASELINE configs[2] launch shape (1184 trees x 128 threads), a few iterations."""
+    root = orc.gen_positions(12, 1, 20, 30)
+    res = mcts.search(root, iterations=3, n_trees=1184, threads_per_tree=128, seed=1000)
+    ostats, obest, _ = orc.uct_search(root, 1184, 128, 3, 1000)
+    _cmp_search(res, ostats, obest)
+
+
+def test_search_async_tree_id_base_merge_identity(mcts, orc):
+    """sum over r of search(tree_id_base = r*n, n trees) == search(0, k*n trees)."""
+    root = orc.gen_positions(13, 1, 20, 40)
+    n, k = 37, 4
+    whole = mcts.search(root, iterations=15, n_trees=n * k, threads_per_tree=64, seed=9)
+    acc = torch.zeros(198, dtype=torch.int64, device="cuda")
+    part = torch.zeros(198, dtype=torch.int64, device="cuda")
+    for r in range(k):
+        mcts.search_async(root, 15, 0.0, n, 64, 9, r * n, part.data_ptr(), torch.cuda.current_stream())
+        acc += part
+    torch.cuda.synchronize()
+    assert acc.cpu().numpy().tolist() == whole["stats"].tolist()
+    ostats, _, _ = orc.uct_search(root, n, 64, 15, 9, tree_id_base=2 * n)
+    mcts.search_async(root, 15, 0.0, n, 64, 9, 2 * n, part.data_ptr(), torch.cuda.current_stream())
+    torch.cuda.synchronize()
+    assert part.cpu().numpy()[:197].tolist() == ostats[:197].tolist()
+
+
+def test_search_leaf_bit_exact(mcts_leaf, orc):
+    root = orc.gen_positions(14, 1, 20, 40)
+    res = mcts_leaf.search(root, iterations=12, n_trees=1, threads_per_tree=1024, seed=3)
+    ostats, obest, oplies = orc.uct_search(root, 1, 1024, 12, 3)
+    _cmp_search(res, ostats, obest)
+    assert res["plies"] == oplies
+
+
+def test_search_leaf_config3_shape(mcts_leaf, orc):
+    """BASELINE configs[3] batch: 16384 threads from one leaf, 2 iterations."""
+    root = orc.gen_positions(15, 1, 30, 40)
+    res = mcts_leaf.search(root, iterations=2, n_trees=1, threads_per_tree=16384, seed=4)
+    ostats, obest, _ = orc.uct_search(root, 1, 16384, 2, 4)
+    _cmp_search(res, ostats, obest)
+
+
+def test_search_terminal_and_pass_roots(mcts, orc):
+    full_black = (1 << 40) - 1
+    full_white = ((1 << 64) - 1) & ~full_black
+    res = mcts.search(orc.position(full_black, full_white, 0), iterations=5, n_trees=3, threads_per_tree=32, seed=1)
+    assert res["best_move"] == -1 and (res["stats"] == 0).all()
+    root = orc.position(0b11, 0b100, 1)
+    res = mcts.search(root, iterations=3, n_trees=2, threads_per_tree=32, seed=1)
+    ostats, obest, _ = orc.uct_search(root, 2, 32, 3, 1)
+    _cmp_search(res, ostats, obest)
+    assert res["best_move"] == 64
+
+
+def test_search_time_mode_invariants(mcts, orc):
+    root = orc.gen_positions(16, 1, 10, 20)
+    res = mcts.search(root, time_ms=50.0, n_trees=148, threads_per_tree=128, seed=5)
+    s = res["stats"]
+    assert res["iterations"] > 148
+    assert s[195] == res["iterations"] * 128
+    assert s[:65].sum() == s[195]
+    assert (s[65:130] + s[130:195] <= s[:65]).all()
+    own, opp = pkg.own_opp(root)
+    legal = orc.legal(own, opp)
+    assert (legal >> res["best_move"]) & 1
+
+
+def test_search_time_mode_pool_full(orc):
+    """A tiny node pool fills up; the search keeps simulating without expanding."""
+    m = pkg.Mcts(c_uct=1.0, scheme="block", max_nodes_per_tree=64, device=0)
+    root = orc.gen_positions(17, 1, 20, 30)
+    res = m.search(root, time_ms=20.0, n_trees=16, threads_per_tree=64, seed=5)
+    s = res["stats"]
+    assert s[195] == res["iterations"] * 64 and s[:65].sum() == s[195]
+    m.close()
+
+
+def test_search_invalid_arguments(mcts, orc):
+    root = orc.opening()
+    for kw in [dict(iterations=0, time_ms=0.0), dict(iterations=5, time_ms=5.0)]:
+        with pytest.raises(pkg.MctsError) as ei:
+            mcts.search(root, n_trees=1, threads_per_tree=32, seed=1, **kw)
+        assert ei.value.status == -1
+    for n_trees, threads in [(0, 32), (1, 48), (1, 2048), (1, 0)]:
+        with pytest.raises(pkg.MctsError):
+            mcts.search(root, iterations=2, n_trees=n_trees, threads_per_tree=threads, seed=1)
+    with pytest.raises(pkg.MctsError) as ei:
+        mcts.search(orc.position(3, 1, 0), iterations=2, n_trees=1, threads_per_tree=32, seed=1)
+    assert ei.value.status == -2
