@@ -129,7 +129,15 @@ def cpu_baseline(budget_s=12.0):
             "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)"}
 
 
+def log(*a):
+    if os.environ.get("BENCH_DEBUG"):
+        print("[bench]", *a, file=sys.stderr, flush=True)
+
+
 def main():
+    if os.environ.get("BENCH_DEBUG"):
+        import faulthandler
+        faulthandler.dump_traceback_later(90, repeat=True)
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
@@ -189,6 +197,7 @@ def main():
         m.playouts_async(d_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, leaf_base,
                          d_out.data_ptr(), d_plies.data_ptr(), stream)
 
+    log('for _ in range(args.warmup):\n ')
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
@@ -216,6 +225,7 @@ def main():
     value = playouts_total / (t_ms / 1e3)
     ms_per_step = t_ms / args.steps
 
+    log('# ---- end to end')
     # ---- end to end through the C ABI with host buffers (H2D + kernel + D2H)
     from paper_conf_ipps_rockis11_b200.positions import own_opp  # noqa: F401
     h_leaves = torch.empty((N_LEAVES, 3), dtype=torch.int64).pin_memory()
@@ -232,6 +242,7 @@ def main():
     barrier()
     e2e_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_s
 
+    log('# ---- block-parallel search')
     # ---- block-parallel search, configs[2] shape, time mode, + root allreduce
     search = None
     leaf_search = None
@@ -261,6 +272,7 @@ def main():
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
         }
+        log('ml = pkg.Mcts(')
         ml = pkg.Mcts(c_uct=1.0, scheme="leaf", device=local)
         lstats = torch.zeros(198, dtype=torch.int64, device="cuda")
         ml.search_async(root, 0, 20.0, 1, LEAF_THREADS, 1000, rank, lstats.data_ptr(), stream)
@@ -281,6 +293,7 @@ def main():
         }
         ml.close()
 
+    log('if sampler is not None:')
     if sampler is not None:
         sampler.terminate()
         sampler.wait()
@@ -327,6 +340,7 @@ def main():
         "clocks": clocks,
         "search": search, "leaf_search": leaf_search,
     }
+    log('if not args.no_cpu and world =')
     if not args.no_cpu and world == 1:
         try:
             line["cpu_baseline"] = cpu_baseline()

@@ -9,6 +9,7 @@
 //   gen_positions_kernel synthetic input recipe
 #pragma once
 #include <cstdint>
+#include <cooperative_groups.h>
 #include "reversi_device.cuh"
 #include "ln_device.cuh"
 #include "tree_device.cuh"
@@ -90,7 +91,7 @@ struct SearchArgs {
   u32 max_iterations;    // iteration budget, or the time-mode cap
   u32 tree_id_base;
   u32 unit;              // playouts per iteration per tree
-  int* error;            // set on a watchdog bailout
+  int* error;            // reserved error flag (0 = ok)
 };
 
 constexpr int kSearchThreadsMax = 1024;
@@ -175,136 +176,87 @@ block_search_kernel(TreePool T, SearchArgs a) {
 
 // ---------------------------------------------------------------------------
 // Leaf-parallel UCT: one tree; every thread of the grid
-// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree.
-// One gather/release barrier per iteration: CTAs add their counts and arrive,
-// CTA 0 waits for all arrivals, backpropagates, selects the next leaf and
-// releases the grid by bumping a generation word. All CTAs are co-resident
-// (cooperative launch); spins carry a watchdog so a fault cannot hang the GPU.
+// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree
+// (select/expand/backprop); the leaf is published through a small global
+// struct between two cooperative-groups grid barriers per iteration
+// (select -> sync -> simulate + per-CTA ballot reduce + atomics -> sync).
+// All CTAs are co-resident (cooperative launch).
 // ---------------------------------------------------------------------------
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
-  u32 gen;          // released iteration + 1
-  u32 arrive;       // cumulative CTA arrivals
   u32 wd[2][2];     // per-iteration-parity wins, draws
 };
 
-__device__ __forceinline__ u32 ld_acquire(const u32* p) {
-  u32 v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release(u32* p, u32 v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-constexpr u64 kWatchdogNs = 120ULL * 1000000000ULL;
-
 __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
   __shared__ u32 path[kMaxPath];
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
-  __shared__ u32 s_go;
   __shared__ u32 s_w[4], s_d[4];
-  __shared__ u64 s_own, s_opp;
-  __shared__ u32 s_term;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const u32 G = gridDim.x;
-  const bool leader_cta = blockIdx.x == 0;
+  const bool leader = blockIdx.x == 0 && warp == 0;
   const u32 unit = a.unit;
-  const u64 start = globaltimer_ns();
   const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
-
-  if (leader_cta && tid == 0) {
+  if (blockIdx.x == 0 && tid == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
     const u64 opp = a.root.to_move ? a.root.black : a.root.white;
     init_node(T, 0, own, opp, 0xFFu);
     s_slot_used = 1;
   }
   __syncthreads();
-  const bool root_term = leader_cta ? meta_term(T.meta[0]) : false;
-
   u32 plies = 0;
   u32 it = 0;
   for (;; ++it) {
-    if (leader_cta && warp == 0) {
+    if (leader) {
       if (it > 0) {
-        // wait for all CTAs of iteration it-1, then backprop
-        if (lane == 0) {
-          const u32 want = G * it;
-          while (ld_acquire(&S->arrive) < want) {
-            if (globaltimer_ns() - start > kWatchdogNs) { atomicExch(a.error, 1); break; }
-          }
-        }
-        __syncwarp();
         const u32 par = (it - 1) & 1u;
-        u32 W = 0, D = 0;
-        if (lane == 0) {
-          W = *((volatile u32*)&S->wd[par][0]);
-          D = *((volatile u32*)&S->wd[par][1]);
-          S->wd[par][0] = 0; S->wd[par][1] = 0;
-        }
-        W = __shfl_sync(kFull, W, 0);
-        D = __shfl_sync(kFull, D, 0);
+        const u32 W = S->wd[par][0], D = S->wd[par][1];
+        __syncwarp();
+        if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
         backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
       }
       u32 stop = 0;
       if (lane == 0) {
-        stop = root_term || it >= a.max_iterations || *((volatile int*)a.error) != 0;
+        stop = meta_term(T.meta[0]) || it >= a.max_iterations;
         if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
       }
       stop = __shfl_sync(kFull, stop, 0);
       if (!stop) {
         const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
-        if (lane == 0) {
-          s_depth = L.depth;
-          S->own = L.own; S->opp = L.opp; S->term = L.term;
-        }
+        if (lane == 0) { s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term; }
       }
-      if (lane == 0) {
-        S->stop = stop;
-        __threadfence();
-        st_release(&S->gen, it + 1);
-      }
+      if (lane == 0) S->stop = stop;
     }
-    // every CTA: wait for the release of iteration `it`
-    if (tid == 0) {
-      while (ld_acquire(&S->gen) < it + 1) {
-        if (globaltimer_ns() - start > kWatchdogNs) { atomicExch(a.error, 1); break; }
-      }
-      s_go = *((volatile u32*)&S->stop) == 0u && *((volatile int*)a.error) == 0;
-      s_own = *((volatile u64*)&S->own);
-      s_opp = *((volatile u64*)&S->opp);
-      s_term = *((volatile u32*)&S->term);
-    }
-    __syncthreads();
-    if (!s_go) break;
+    grid.sync();
+    const u32 stop = S->stop;
+    const u64 own = S->own, opp = S->opp;
+    const u32 term = S->term;
+    if (stop) break;
     int r;
-    if (s_term) {
-      const int x = __popcll(s_own), y = __popcll(s_opp);
+    if (term) {
+      const int x = __popcll(own), y = __popcll(opp);
       r = (x > y) - (x < y);
     } else {
-      r = playout(s_own, s_opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, &plies);
+      r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, &plies);
     }
     const u32 bw = __popc(__ballot_sync(kFull, r == 1));
     const u32 bd = __popc(__ballot_sync(kFull, r == 0));
     if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
     __syncthreads();
     if (tid == 0) {
-      const u32 W = s_w[0] + s_w[1] + s_w[2] + s_w[3];
-      const u32 D = s_d[0] + s_d[1] + s_d[2] + s_d[3];
       const u32 par = it & 1u;
-      if (W) atomicAdd(&S->wd[par][0], W);
-      if (D) atomicAdd(&S->wd[par][1], D);
-      __threadfence();
-      atomicAdd(&S->arrive, 1u);
+      atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
+      atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
     }
+    grid.sync();
   }
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
-  if (leader_cta && warp == 0) merge_root(T, 0, unit, it, a.stats, lane);
+  if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
 
 // ---------------------------------------------------------------------------

@@ -228,14 +228,15 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
   // leaf parallelism: one cooperative grid of unit/128 co-resident CTAs
   const uint32_t G = threads_per_tree / 128;
   int per_sm = 0, n_sm = 0;
-  CK(h, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, leaf_search_kernel, 128, 0));
+  const void* kfn = (const void*)leaf_search_kernel;
+  CK(h, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, 128, 0));
   CK(h, cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, h->device));
   if ((long long)per_sm * n_sm < (long long)G)
     return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: batch does not fit co-resident on the device");
   CK(h, cudaMemsetAsync(h->d_leafsync, 0, sizeof(LeafSync), s));
   LeafSync* S = h->d_leafsync;
   void* args[] = {(void*)&T, (void*)&a, (void*)&S};
-  CK(h, cudaLaunchCooperativeKernel((const void*)leaf_search_kernel, dim3(G), dim3(128), args, 0, s));
+  CK(h, cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(128), args, 0, s));
   return MCTS_OK;
 }
 
@@ -402,7 +403,7 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   int herr = 0;
   CK(h, cudaMemcpyAsync(&herr, h->d_error, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CK(h, cudaStreamSynchronize(h->stream));
-  if (herr) return fail(h, MCTS_E_CUDA, "leaf search watchdog fired (grid barrier did not complete)");
+  if (herr) return fail(h, MCTS_E_CUDA, "search kernel reported an internal error");
   for (int i = 0; i < 65; ++i) {
     out->visits[i] = (uint64_t)hs[i];
     out->wins[i] = (uint64_t)hs[65 + i];

@@ -77,7 +77,8 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
   if (lane == 0) path[0] = 0;
   u32 meta = T.meta[base];
   // Selection (L157-L178): descend while the node is non-terminal and fully expanded.
-  while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta)) {
+  // (depth bound: a game has < 128 plies incl. passes; never reached)
+  while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta) && depth < kMaxPath - 2) {
     const u32 nch = meta_nchild(meta);
     const u32 first = T.first[base + v];
     const double lnp = lnT[T.k[base + v]];
