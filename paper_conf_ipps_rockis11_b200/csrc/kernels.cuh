@@ -43,6 +43,9 @@ constexpr int kPlayoutThreads = 128;
 __global__ void __launch_bounds__(kPlayoutThreads)
 playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
                 u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out) {
+  __shared__ u64 s_rays[256];
+  fill_rays(s_rays);
+  __syncthreads();
   const u64 g = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   const u64 total = (u64)n_leaves * n_per_leaf;
   const bool active = g < total;
@@ -55,7 +58,7 @@ playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_
     const DevPosition p = leaves[leaf];
     const u64 own = p.to_move ? p.white : p.black;
     const u64 opp = p.to_move ? p.black : p.white;
-    r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, &plies);
+    r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, s_rays, &plies);
   }
   const int lane = threadIdx.x & 31;
   const u32 grp = __match_any_sync(kFull, leaf);
@@ -104,6 +107,8 @@ block_search_kernel(TreePool T, SearchArgs a) {
   __shared__ u32 s_term, s_stop, s_slot_used;
   __shared__ u32 s_w[32], s_d[32];
   __shared__ int s_depth;
+  __shared__ u64 s_rays[256];
+  fill_rays(s_rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nwarps = blockDim.x >> 5;
@@ -147,7 +152,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
         const int x = __popcll(s_own), y = __popcll(s_opp);
         r = (x > y) - (x < y);
       } else {
-        r = playout(s_own, s_opp, a.key, c0, it, (u32)tid, &plies);
+        r = playout(s_own, s_opp, a.key, c0, it, (u32)tid, s_rays, &plies);
       }
       const u32 bw = __popc(__ballot_sync(kFull, r == 1));
       const u32 bd = __popc(__ballot_sync(kFull, r == 0));
@@ -196,6 +201,8 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
   __shared__ u32 s_w[4], s_d[4];
+  __shared__ u64 s_rays[256];
+  fill_rays(s_rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const bool leader = blockIdx.x == 0 && warp == 0;
@@ -241,7 +248,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       const int x = __popcll(own), y = __popcll(opp);
       r = (x > y) - (x < y);
     } else {
-      r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, &plies);
+      r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, s_rays, &plies);
     }
     const u32 bw = __popc(__ballot_sync(kFull, r == 1));
     const u32 bd = __popc(__ballot_sync(kFull, r == 0));

@@ -108,12 +108,13 @@ __device__ __forceinline__ u64 legal_moves_fast(u64 P, u64 O) {
 // Upward ray masks (squares strictly beyond sq in direction +1, +8, +7, +9 up
 // to the board edge), one table of 4 x 64 u64 per CTA in shared memory.
 __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
-  const int dr[4] = {0, 1, 1, 1}, dc[4] = {1, 0, -1, 1};
+  const int dr = dir_index == 0 ? 0 : 1;
+  const int dc = dir_index == 1 ? 0 : (dir_index == 2 ? -1 : 1);
   int r = sq >> 3, c = sq & 7;
   u64 m = 0;
   for (;;) {
-    r += dr[dir_index];
-    c += dc[dir_index];
+    r += dr;
+    c += dc;
     if (r < 0 || r > 7 || c < 0 || c > 7) break;
     m |= 1ULL << (8 * r + c);
   }
@@ -209,7 +210,7 @@ struct PlayoutRng {
 // to move at the start (R3), adds the non-pass plies to *plies.
 // A pass consumes no RNG word; two consecutive passes end the game.
 __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1, u32 c2,
-                                       u32* plies) {
+                                       const u64* __restrict__ rays, u32* plies) {
   PlayoutRng rng;
   rng.key = key; rng.c0 = c0; rng.c1 = c1; rng.c2 = c2; rng.w = 0;
   rng.buf = make_uint4(0, 0, 0, 0);
@@ -217,14 +218,14 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   bool passed = false;
   u32 n = 0;
   for (;;) {
-    const u64 moves = legal_moves(me, op);
+    const u64 moves = legal_moves_fast(me, op);
     if (moves == 0ULL) {
       if (passed) break;  // neither player can move
       passed = true;
     } else {
       passed = false;
       const int sq = pick_square(moves, rng.next());
-      const u64 f = flips(sq, me, op);
+      const u64 f = flips_fast(sq, me, op, rays);
       me |= f | (1ULL << sq);
       op &= ~f;
       ++n;
@@ -235,6 +236,12 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   *plies += n;
   const int a = __popcll(start ? me : op), b = __popcll(start ? op : me);
   return (a > b) - (a < b);
+}
+
+// Fill the per-CTA shared ray table (4 x 64 u64) used by flips_fast; every
+// thread of the block must call it, followed by __syncthreads().
+__device__ __forceinline__ void fill_rays(u64* rays) {
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) rays[i] = ray_mask(i >> 6, i & 63);
 }
 
 // Terminal test: neither side has a move.
