@@ -43,7 +43,7 @@ constexpr int kPlayoutThreads = 128;
 __global__ void __launch_bounds__(kPlayoutThreads)
 playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
                 u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out) {
-  __shared__ u64 s_rays[256];
+  __shared__ u64 s_rays[kRayTable];
   fill_rays(s_rays);
   __syncthreads();
   const u64 g = (u64)blockIdx.x * blockDim.x + threadIdx.x;
@@ -107,7 +107,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
   __shared__ u32 s_term, s_stop, s_slot_used;
   __shared__ u32 s_w[32], s_d[32];
   __shared__ int s_depth;
-  __shared__ u64 s_rays[256];
+  __shared__ u64 s_rays[kRayTable];
   fill_rays(s_rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -201,7 +201,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
   __shared__ u32 s_w[4], s_d[4];
-  __shared__ u64 s_rays[256];
+  __shared__ u64 s_rays[kRayTable];
   fill_rays(s_rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;

@@ -76,37 +76,81 @@ __device__ __forceinline__ u64 flips(int sq, u64 P, u64 O) {
 }
 
 // ---------------------------------------------------------------------------
-// Faster variants (same results, fewer issue slots).
+// Hot-loop variants (same results as legal_moves / flips, fewer ALU-pipe slots).
 //
+// The playout loop is integer-issue bound and, compiled naively, saturates the
+// ALU pipe (LOP3/SHF/IADD3/SEL, 16 lanes/SMSP/clk) while the FMA pipe (IMAD,
+// also 16 lanes/SMSP/clk) idles. Shifting by multiplying with a power of two
+// runs on the FMA pipe; the multipliers live in constant memory so ptxas cannot
+// fold them back into SHF. Each shift helper picks its pipe mix by template
+// argument:
+//   shl<S, kAlu>: IMAD.SHL + SHF        shl<S, kFma>: IMAD.WIDE + IMAD
+//   shr<S, kAlu>: 2 x SHF               shr<S, kMix>: SHF + IMAD.HI
+//   shr<S, kFma>: IMAD.HI + IMAD + IMAD.HI
+__constant__ u32 c_pow2[33] = {
+    1u, 2u, 4u, 8u, 16u, 32u, 64u, 128u, 256u, 512u, 1024u, 2048u, 4096u, 8192u, 16384u, 32768u,
+    1u << 16, 1u << 17, 1u << 18, 1u << 19, 1u << 20, 1u << 21, 1u << 22, 1u << 23, 1u << 24,
+    1u << 25, 1u << 26, 1u << 27, 1u << 28, 1u << 29, 1u << 30, 1u << 31, 0u};
+
+enum { kAlu = 0, kFma = 1, kMix = 2 };
+
+__device__ __forceinline__ u64 join32(u32 lo, u32 hi) { return ((u64)hi << 32) | lo; }
+
+template <int S, int MODE>
+__device__ __forceinline__ u64 shl(u64 x) {
+  static_assert(S > 0 && S < 32, "shift");
+  if constexpr (MODE == kAlu) {
+    return x << S;
+  } else {
+    const u32 lo = (u32)x, hi = (u32)(x >> 32), m = c_pow2[S];
+    return join32(lo * m, hi * m + __umulhi(lo, m));
+  }
+}
+
+template <int S, int MODE>
+__device__ __forceinline__ u64 shr(u64 x) {
+  static_assert(S > 0 && S < 32, "shift");
+  const u32 lo = (u32)x, hi = (u32)(x >> 32);
+  if constexpr (MODE == kAlu) {
+    return x >> S;
+  } else if constexpr (MODE == kMix) {
+    return join32(__funnelshift_r(lo, hi, S), __umulhi(hi, c_pow2[32 - S]));
+  } else {
+    const u32 m = c_pow2[32 - S];
+    return join32(hi * m + __umulhi(lo, m), __umulhi(hi, m));
+  }
+}
+
 // Move generation with a shared doubled propagator: after two single steps the
 // run from P covers 2 squares, after two double steps (M2 = M & M<<S) it covers
 // 6, the longest possible run. M2 for -S is M2 >> S, so an axis costs one M2.
-template <int S>
+template <int S, int LM, int RM>
 __device__ __forceinline__ u64 axis_moves(u64 P, u64 M) {
-  const u64 M2 = M & sh<S>(M);
-  u64 t = M & sh<S>(P);
-  t |= M & sh<S>(t);
-  t |= M2 & sh<2 * S>(t);
-  t |= M2 & sh<2 * S>(t);
-  const u64 M2r = sh<-S>(M2);
-  u64 u = M & sh<-S>(P);
-  u |= M & sh<-S>(u);
-  u |= M2r & sh<-2 * S>(u);
-  u |= M2r & sh<-2 * S>(u);
-  return sh<S>(t) | sh<-S>(u);
+  const u64 M2 = M & shl<S, LM>(M);
+  u64 t = M & shl<S, LM>(P);
+  t |= M & shl<S, LM>(t);
+  t |= M2 & shl<2 * S, LM>(t);
+  t |= M2 & shl<2 * S, LM>(t);
+  const u64 M2r = shr<S, RM>(M2);
+  u64 u = M & shr<S, RM>(P);
+  u |= M & shr<S, RM>(u);
+  u |= M2r & shr<2 * S, RM>(u);
+  u |= M2r & shr<2 * S, RM>(u);
+  return shl<S, LM>(t) | shr<S, RM>(u);
 }
 
 __device__ __forceinline__ u64 legal_moves_fast(u64 P, u64 O) {
   const u64 M = O & kInner;
-  u64 m = axis_moves<1>(P, M);
-  m |= axis_moves<8>(P, O);
-  m |= axis_moves<7>(P, M);
-  m |= axis_moves<9>(P, M);
+  u64 m = axis_moves<1, kFma, kMix>(P, M);
+  m |= axis_moves<8, kFma, kFma>(P, O);
+  m |= axis_moves<7, kFma, kMix>(P, M);
+  m |= axis_moves<9, kFma, kFma>(P, M);
   return m & ~(P | O);
 }
 
 // Upward ray masks (squares strictly beyond sq in direction +1, +8, +7, +9 up
-// to the board edge), one table of 4 x 64 u64 per CTA in shared memory.
+// to the board edge) and the ray's first square, in a per-CTA shared table:
+// rays[d*64 + sq] = mask, rays[256 + d*64 + sq] = first square (0 at an edge).
 __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
   const int dr = dir_index == 0 ? 0 : 1;
   const int dc = dir_index == 1 ? 0 : (dir_index == 2 ? -1 : 1);
@@ -121,32 +165,38 @@ __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
   return m;
 }
 
-// Flips along an upward direction by carry propagation: adding the first ray
-// square to (O | ~m) carries through the contiguous opponent run (and through
-// the non-ray bits, all ones) and lands on the first non-opponent ray square.
-// run = ray squares that carried (~s & O & m); valid iff the landing square is P.
-template <int S>
-__device__ __forceinline__ u64 up_flips(u64 x, u64 P, u64 O, u64 m) {
-  const u64 s = (O | ~m) + sh<S>(x);
-  const u64 run = ~s & O & m;
-  return (s & m & P) ? run : 0ULL;
+constexpr int kRayTable = 512;
+
+// Flips along an upward ray by carry propagation: adding the ray's first square
+// to (O | ~m) carries through the contiguous opponent run (and through the
+// non-ray bits, all ones) and lands on the first non-opponent ray square.
+// run = ray squares that carried (~s & O & m); kept iff the landing square is P.
+// The 64-bit add runs on the FMA pipe (IMAD.WIDE by one, then IMAD on the high
+// word: first is a single bit, so at most one of its halves is non-zero).
+__device__ __forceinline__ void up_flips(u64& f, u64 first, u64 P, u64 O, u64 m, u32 one) {
+  const u64 xo = O | ~m;
+  const u64 s0 = (u64)((u32)first) * one + xo;
+  const u64 s = join32((u32)s0, (u32)(first >> 32) * one + (u32)(s0 >> 32));
+  if (s & m & P) f |= ~s & O & m;
 }
 
 // All 8 directions: the 4 upward ones directly, the 4 downward ones as upward
 // directions of the 180-degree-rotated (bit-reversed) board, where square sq
-// becomes 63 - sq and the same ray table applies.
+// becomes 63 - sq and the same table applies.
 __device__ __forceinline__ u64 flips_fast(int sq, u64 P, u64 O, const u64* __restrict__ rays) {
-  const u64 x = 1ULL << sq;
-  u64 f = up_flips<1>(x, P, O, rays[sq]);
-  f |= up_flips<8>(x, P, O, rays[64 + sq]);
-  f |= up_flips<7>(x, P, O, rays[128 + sq]);
-  f |= up_flips<9>(x, P, O, rays[192 + sq]);
+  const u32 one = c_pow2[0];
+  u64 f = 0;
+  up_flips(f, rays[256 + sq], P, O, rays[sq], one);
+  up_flips(f, rays[320 + sq], P, O, rays[64 + sq], one);
+  up_flips(f, rays[384 + sq], P, O, rays[128 + sq], one);
+  up_flips(f, rays[448 + sq], P, O, rays[192 + sq], one);
   const int rs = 63 - sq;
-  const u64 rx = 1ULL << rs, rP = __brevll(P), rO = __brevll(O);
-  u64 g = up_flips<1>(rx, rP, rO, rays[rs]);
-  g |= up_flips<8>(rx, rP, rO, rays[64 + rs]);
-  g |= up_flips<7>(rx, rP, rO, rays[128 + rs]);
-  g |= up_flips<9>(rx, rP, rO, rays[192 + rs]);
+  const u64 rP = __brevll(P), rO = __brevll(O);
+  u64 g = 0;
+  up_flips(g, rays[256 + rs], rP, rO, rays[rs], one);
+  up_flips(g, rays[320 + rs], rP, rO, rays[64 + rs], one);
+  up_flips(g, rays[384 + rs], rP, rO, rays[128 + rs], one);
+  up_flips(g, rays[448 + rs], rP, rO, rays[192 + rs], one);
   return f | __brevll(g);
 }
 
@@ -241,7 +291,11 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
 // Fill the per-CTA shared ray table (4 x 64 u64) used by flips_fast; every
 // thread of the block must call it, followed by __syncthreads().
 __device__ __forceinline__ void fill_rays(u64* rays) {
-  for (int i = threadIdx.x; i < 256; i += blockDim.x) rays[i] = ray_mask(i >> 6, i & 63);
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) {
+    const u64 m = ray_mask(i >> 6, i & 63);
+    rays[i] = m;
+    rays[256 + i] = m & (0ULL - m);  // lowest ray square (0 if the ray is empty)
+  }
 }
 
 // Terminal test: neither side has a move.
