@@ -32,43 +32,61 @@ __device__ __forceinline__ u64 globaltimer_ns() {
 }
 
 // ---------------------------------------------------------------------------
-// Batched playouts. Thread g plays playout j = g mod n_per_leaf of leaf
-// g / n_per_leaf (leaf-major, so the 32 lanes of a warp usually share a leaf
-// and finish within a ply or two of each other). Outcomes are reduced per
-// (warp, leaf) with match_any + ballot + popc and added with one atomic per
-// counter; the ply count with one atomic per warp.
+// Batched playouts, persistent: the grid is sized to the resident capacity and
+// each warp repeatedly takes the next chunk of 32 playouts from a work counter
+// (dynamic balancing; the per-CTA ray table is loaded once). Playout g of a
+// launch is playout j = g mod n_per_leaf of leaf g / n_per_leaf (leaf-major, so
+// a warp's 32 lanes usually share a leaf and finish within a ply or two of each
+// other). Outcomes are reduced per (warp, leaf) with match_any + ballot + popc
+// and added with one atomic per counter; plies with one atomic per warp.
 // ---------------------------------------------------------------------------
 constexpr int kPlayoutThreads = 128;
 
+__global__ void rays_init_kernel(u64* g_rays) {
+  fill_rays(g_rays);
+}
+
+__device__ __forceinline__ void load_rays(u64* s_rays, const u64* __restrict__ g_rays) {
+  for (int i = threadIdx.x; i < kRayTable; i += blockDim.x) s_rays[i] = g_rays[i];
+}
+
 __global__ void __launch_bounds__(kPlayoutThreads)
 playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
-                u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out) {
+                u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out,
+                const u64* __restrict__ g_rays, u32* __restrict__ work) {
   __shared__ u64 s_rays[kRayTable];
-  fill_rays(s_rays);
+  load_rays(s_rays, g_rays);
   __syncthreads();
-  const u64 g = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   const u64 total = (u64)n_leaves * n_per_leaf;
-  const bool active = g < total;
-  u32 leaf = 0xFFFFFFFFu, j = 0;
-  int r = 2;
-  u32 plies = 0;
-  if (active) {
-    leaf = (u32)(g / n_per_leaf);
-    j = (u32)(g - (u64)leaf * n_per_leaf);
-    const DevPosition p = leaves[leaf];
-    const u64 own = p.to_move ? p.white : p.black;
-    const u64 opp = p.to_move ? p.black : p.white;
-    r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, s_rays, &plies);
-  }
+  const u32 n_chunks = (u32)((total + 31) / 32);
   const int lane = threadIdx.x & 31;
-  const u32 grp = __match_any_sync(kFull, leaf);
-  const u32 wins = __popc(__ballot_sync(kFull, r == 1) & grp);
-  const u32 draws = __popc(__ballot_sync(kFull, r == 0) & grp);
-  const u32 losses = __popc(__ballot_sync(kFull, r == -1) & grp);
-  if (active && lane == __ffs(grp) - 1) {
-    if (wins) atomicAdd(&out[leaf].wins, wins);
-    if (draws) atomicAdd(&out[leaf].draws, draws);
-    if (losses) atomicAdd(&out[leaf].losses, losses);
+  u32 plies = 0;
+  for (;;) {
+    u32 chunk = 0;
+    if (lane == 0) chunk = atomicAdd(work, 1u);
+    chunk = __shfl_sync(kFull, chunk, 0);
+    if (chunk >= n_chunks) break;
+    const u64 g = (u64)chunk * 32u + (u32)lane;
+    const bool active = g < total;
+    u32 leaf = 0xFFFFFFFFu;
+    int r = 2;
+    if (active) {
+      leaf = (u32)(g / n_per_leaf);
+      const u32 j = (u32)(g - (u64)leaf * n_per_leaf);
+      const DevPosition p = leaves[leaf];
+      const u64 own = p.to_move ? p.white : p.black;
+      const u64 opp = p.to_move ? p.black : p.white;
+      r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, s_rays, &plies);
+    }
+    const u32 grp = __match_any_sync(kFull, leaf);
+    const u32 wins = __popc(__ballot_sync(kFull, r == 1) & grp);
+    const u32 draws = __popc(__ballot_sync(kFull, r == 0) & grp);
+    const u32 losses = __popc(__ballot_sync(kFull, r == -1) & grp);
+    if (active && lane == __ffs(grp) - 1) {
+      if (wins) atomicAdd(&out[leaf].wins, wins);
+      if (draws) atomicAdd(&out[leaf].draws, draws);
+      if (losses) atomicAdd(&out[leaf].losses, losses);
+    }
   }
   if (plies_out) {
     const u32 s = __reduce_add_sync(kFull, plies);
@@ -95,6 +113,7 @@ struct SearchArgs {
   u32 tree_id_base;
   u32 unit;              // playouts per iteration per tree
   int* error;            // reserved error flag (0 = ok)
+  const u64* rays;       // global ray table (kRayTable u64)
 };
 
 constexpr int kSearchThreadsMax = 1024;
@@ -108,7 +127,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
   __shared__ u32 s_w[32], s_d[32];
   __shared__ int s_depth;
   __shared__ u64 s_rays[kRayTable];
-  fill_rays(s_rays);
+  load_rays(s_rays, a.rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nwarps = blockDim.x >> 5;
@@ -202,7 +221,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   __shared__ int s_depth;
   __shared__ u32 s_w[4], s_d[4];
   __shared__ u64 s_rays[kRayTable];
-  fill_rays(s_rays);
+  load_rays(s_rays, a.rays);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const bool leader = blockIdx.x == 0 && warp == 0;

@@ -51,6 +51,9 @@ struct mcts_handle {
   unsigned long long* d_t0 = nullptr;
   int* d_error = nullptr;
   LeafSync* d_leafsync = nullptr;
+  u64* d_rays = nullptr;      // ray table for the flip kernels (kRayTable u64)
+  u32* d_work = nullptr;      // playout work counter
+  int playout_ctas = 0;       // resident playout CTAs (SMs x occupancy)
 };
 
 namespace {
@@ -214,6 +217,7 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
   a.tree_id_base = tree_id_base;
   a.unit = (u32)unit;
   a.error = h->d_error;
+  a.rays = h->d_rays;
   if (by_time) {
     stamp_kernel<<<1, 1, 0, s>>>(h->d_t0);
     CK(h, cudaGetLastError());
@@ -293,6 +297,18 @@ mcts_status mcts_create(const mcts_position* position, const mcts_params* params
   if (e == cudaSuccess) e = cudaMalloc(&h->d_error, sizeof(int));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_plies, sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_leafsync, sizeof(LeafSync));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_rays, kRayTable * sizeof(u64));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_work, sizeof(u32));
+  if (e == cudaSuccess) {
+    rays_init_kernel<<<1, 256, 0, h->stream>>>(h->d_rays);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess) {
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, playouts_kernel, kPlayoutThreads, 0);
+    h->playout_ctas = per_sm * prop.multiProcessorCount;
+  }
   if (e != cudaSuccess) {
     g_create_error = std::string("mcts_create: ") + cudaGetErrorString(e);
     mcts_destroy(h);
@@ -315,6 +331,8 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_t0);
   cudaFree(h->d_error);
   cudaFree(h->d_leafsync);
+  cudaFree(h->d_rays);
+  cudaFree(h->d_work);
   if (h->h_pinned) cudaFreeHost(h->h_pinned);
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;
@@ -332,11 +350,13 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
   CK(h, cudaMemsetAsync(d_out, 0, (size_t)n_leaves * sizeof(mcts_wdl), s));
   const uint64_t total = (uint64_t)n_leaves * n_per_leaf;
   if (total == 0) return MCTS_OK;
-  const uint64_t blocks = (total + kPlayoutThreads - 1) / kPlayoutThreads;
-  if (blocks > 0x7FFFFFFFull) return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large");
-  playouts_kernel<<<(unsigned)blocks, kPlayoutThreads, 0, s>>>(
+  if ((total + 31) / 32 > 0xFFFFFFF0ull) return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large (>= 2^37 playouts)");
+  const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
+  const unsigned blocks = (unsigned)(need < (uint64_t)h->playout_ctas ? need : (uint64_t)h->playout_ctas);
+  CK(h, cudaMemsetAsync(h->d_work, 0, sizeof(u32), s));
+  playouts_kernel<<<blocks, kPlayoutThreads, 0, s>>>(
       (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), leaf_id_base, (WdlOut*)d_out,
-      (unsigned long long*)d_plies);
+      (unsigned long long*)d_plies, h->d_rays, h->d_work);
   CK(h, cudaGetLastError());
   return MCTS_OK;
 }
