@@ -200,6 +200,96 @@ __device__ __forceinline__ u64 flips_fast(int sq, u64 P, u64 O, const u64* __res
   return f | __brevll(g);
 }
 
+// ---- FMA-pipe integer helpers (the multiplier 1 comes from constant memory
+// so ptxas keeps IMAD rather than an ALU-pipe IADD3) ----------------------------
+__device__ __forceinline__ u32 add_f(u32 a, u32 b) { return a * c_pow2[0] + b; }   // a + b
+__device__ __forceinline__ u32 sub_f(u32 a, u32 b) { return b * (0u - c_pow2[0]) + a; }  // a - b
+// Disjoint 64-bit add / subset subtract as two independent 32-bit IMADs:
+// a | b when a & b == 0, and a & ~b when b is a subset of a.
+__device__ __forceinline__ u64 or_disjoint_f(u64 a, u64 b) {
+  return join32(add_f((u32)a, (u32)b), add_f((u32)(a >> 32), (u32)(b >> 32)));
+}
+__device__ __forceinline__ u64 andnot_subset_f(u64 a, u64 b) {
+  return join32(sub_f((u32)a, (u32)b), sub_f((u32)(a >> 32), (u32)(b >> 32)));
+}
+
+// Horizontal (+1) moves by carry propagation, per 32-bit half (a row never
+// spans halves and no carry leaves a row: the landing square of a run ending
+// on column 6 is column 7, and column 7 is never in M). t = P<<1 per half;
+// s = M + t carries each adjacent opponent run to its landing square; s & ~t
+// keeps landings (and non-carried O / P squares, removed by the final empty
+// mask of the caller).
+__device__ __forceinline__ u64 east_moves_f(u64 P, u64 M) {
+  const u32 two = c_pow2[1];
+  const u32 tl = (u32)P * two, th = (u32)(P >> 32) * two;
+  const u32 sl = add_f((u32)M, tl), sh_ = add_f((u32)(M >> 32), th);
+  return join32(sl & ~tl, sh_ & ~th);
+}
+
+// Legal moves with the horizontal axis done by carries (west as east of the
+// bit-reversed board rP/rO, which the caller also reuses for the flips) and
+// the other three axes by the doubled-propagator fill.
+__device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
+  const u64 M = O & kInner;
+  u64 m = east_moves_f(P, M);
+  m |= axis_moves<8, kFma, kFma>(P, O);
+  m |= axis_moves<7, kFma, kFma>(P, M);
+  m |= axis_moves<9, kFma, kFma>(P, M);
+  m |= __brevll(east_moves_f(rP, rO & kInner));
+  return m & ~(P | O);
+}
+
+// flips_fast with the bit-reversed board supplied by the caller.
+__device__ __forceinline__ u64 flips_hot(int sq, u64 P, u64 O, u64 rP, u64 rO,
+                                         const u64* __restrict__ rays) {
+  const u32 one = c_pow2[0];
+  u64 f = 0;
+  up_flips(f, rays[256 + sq], P, O, rays[sq], one);
+  up_flips(f, rays[320 + sq], P, O, rays[64 + sq], one);
+  up_flips(f, rays[384 + sq], P, O, rays[128 + sq], one);
+  up_flips(f, rays[448 + sq], P, O, rays[192 + sq], one);
+  const int rs = 63 - sq;
+  u64 g = 0;
+  up_flips(g, rays[256 + rs], rP, rO, rays[rs], one);
+  up_flips(g, rays[320 + rs], rP, rO, rays[64 + rs], one);
+  up_flips(g, rays[384 + rs], rP, rO, rays[128 + rs], one);
+  up_flips(g, rays[448 + rs], rP, rO, rays[192 + rs], one);
+  return f | __brevll(g);
+}
+
+// k-th set bit with the selects done arithmetically on the FMA pipe:
+// per level s = (k < c) in {0,1} from the sign of k - c, then
+// x = hi + s*(lo - hi), k = (k - c) + s*c, base += W*(1 - s).
+__device__ __forceinline__ int kth_set_bit_f(u64 m, u32 k) {
+  const u32 one = c_pow2[0];
+  u32 x = (u32)m;
+  const u32 hi = (u32)(m >> 32);
+  u32 c = __popc(x);
+  u32 d = sub_f(k, c);
+  u32 sgn = __umulhi(d, c_pow2[1]);  // (k - c) >> 31: 1 iff k < c
+  x = sgn * (x - hi) + hi;
+  k = sgn * c + d;
+  u32 base = sgn * (0u - 32u * one) + 32u;
+#pragma unroll
+  for (int wdt = 16; wdt >= 2; wdt >>= 1) {
+    const u32 lowm = x & ((1u << wdt) - 1u);
+    c = __popc(lowm);
+    d = sub_f(k, c);
+    sgn = __umulhi(d, c_pow2[1]);
+    // upper part: x >> wdt on the FMA pipe
+    const u32 up = __umulhi(x, c_pow2[32 - wdt]);
+    x = sgn * (lowm - up) + up;
+    k = sgn * c + d;
+    base = sgn * (0u - (u32)wdt * one) + (base + (u32)wdt);
+  }
+  // last level (width 1): bit 0 of x is set iff c = 1
+  c = x & 1u;
+  d = sub_f(k, c);
+  sgn = __umulhi(d, c_pow2[1]);
+  base = sgn * (0u - one) + (base + 1u);
+  return (int)base;
+}
+
 // Index (0..63) of the k-th set bit (k = 0: lowest) of m; k < popc(m).
 // Branch-free binary search on population counts.
 __device__ __forceinline__ int kth_set_bit(u64 m, u32 k) {
@@ -243,15 +333,14 @@ struct PlayoutRng {
   uint2 key;
   u32 c0, c1, c2;
   u32 w;
-  uint4 buf;
+  uint4 buf;  // the unread words of the current Philox block, in order
   __device__ __forceinline__ u32 next() {
-    const u32 lane = w & 3u;
-    if (lane == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
+    if ((w & 3u) == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
     ++w;
-    u32 r = buf.x;
-    r = lane == 1u ? buf.y : r;
-    r = lane == 2u ? buf.z : r;
-    r = lane == 3u ? buf.w : r;
+    const u32 r = buf.x;
+    buf.x = buf.y;
+    buf.y = buf.z;
+    buf.z = buf.w;
     return r;
   }
 };
@@ -268,16 +357,18 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   bool passed = false;
   u32 n = 0;
   for (;;) {
-    const u64 moves = legal_moves_fast(me, op);
+    const u64 rme = __brevll(me), rop = __brevll(op);
+    const u64 moves = legal_moves_hot(me, op, rme, rop);
     if (moves == 0ULL) {
       if (passed) break;  // neither player can move
       passed = true;
     } else {
       passed = false;
-      const int sq = pick_square(moves, rng.next());
-      const u64 f = flips_fast(sq, me, op, rays);
-      me |= f | (1ULL << sq);
-      op &= ~f;
+      const u32 r = rng.next();
+      const int sq = kth_set_bit_f(moves, __umulhi(r, (u32)__popcll(moves)));
+      const u64 f = flips_hot(sq, me, op, rme, rop, rays);
+      me = or_disjoint_f(me, or_disjoint_f(f, 1ULL << sq));
+      op = andnot_subset_f(op, f);
       ++n;
     }
     const u64 t = me; me = op; op = t;
