@@ -40,7 +40,13 @@ __device__ __forceinline__ u64 globaltimer_ns() {
 // other). Outcomes are reduced per (warp, leaf) with match_any + ballot + popc
 // and added with one atomic per counter; plies with one atomic per warp.
 // ---------------------------------------------------------------------------
-constexpr int kPlayoutThreads = 128;
+#ifndef MCTS_PLAYOUT_THREADS
+#define MCTS_PLAYOUT_THREADS 128
+#endif
+#ifndef MCTS_PLAYOUT_MINB
+#define MCTS_PLAYOUT_MINB 1
+#endif
+constexpr int kPlayoutThreads = MCTS_PLAYOUT_THREADS;
 
 __global__ void rays_init_kernel(u64* g_rays) {
   fill_rays(g_rays);
@@ -50,7 +56,7 @@ __device__ __forceinline__ void load_rays(u64* s_rays, const u64* __restrict__ g
   for (int i = threadIdx.x; i < kRayTable; i += blockDim.x) s_rays[i] = g_rays[i];
 }
 
-__global__ void __launch_bounds__(kPlayoutThreads)
+__global__ void __launch_bounds__(kPlayoutThreads, MCTS_PLAYOUT_MINB)
 playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
                 u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out,
                 const u64* __restrict__ g_rays, u32* __restrict__ work) {

@@ -94,6 +94,32 @@ __constant__ u32 c_pow2[33] = {
 
 enum { kAlu = 0, kFma = 1, kMix = 2 };
 
+// Pipe-mix configuration of the hot loop (tuned on B200).
+#ifndef MCTS_MG_LEFT
+#define MCTS_MG_LEFT kAlu
+#endif
+#ifndef MCTS_MG_RIGHT
+#define MCTS_MG_RIGHT kAlu
+#endif
+#ifndef MCTS_MG_EAST_CARRY
+#define MCTS_MG_EAST_CARRY 1
+#endif
+#ifndef MCTS_EAST_PLAIN
+#define MCTS_EAST_PLAIN 0
+#endif
+#ifndef MCTS_PICK_F
+#define MCTS_PICK_F 0
+#endif
+#ifndef MCTS_UPD_F
+#define MCTS_UPD_F 0
+#endif
+#ifndef MCTS_FLIP_ADD_F
+#define MCTS_FLIP_ADD_F 0
+#endif
+#ifndef MCTS_RNG_SELECT
+#define MCTS_RNG_SELECT 0
+#endif
+
 __device__ __forceinline__ u64 join32(u32 lo, u32 hi) { return ((u64)hi << 32) | lo; }
 
 template <int S, int MODE>
@@ -175,8 +201,12 @@ constexpr int kRayTable = 512;
 // word: first is a single bit, so at most one of its halves is non-zero).
 __device__ __forceinline__ void up_flips(u64& f, u64 first, u64 P, u64 O, u64 m, u32 one) {
   const u64 xo = O | ~m;
+#if MCTS_FLIP_ADD_F
   const u64 s0 = (u64)((u32)first) * one + xo;
   const u64 s = join32((u32)s0, (u32)(first >> 32) * one + (u32)(s0 >> 32));
+#else
+  const u64 s = xo + first;
+#endif
   if (s & m & P) f |= ~s & O & m;
 }
 
@@ -220,9 +250,14 @@ __device__ __forceinline__ u64 andnot_subset_f(u64 a, u64 b) {
 // keeps landings (and non-carried O / P squares, removed by the final empty
 // mask of the caller).
 __device__ __forceinline__ u64 east_moves_f(u64 P, u64 M) {
+#if MCTS_EAST_PLAIN
+  const u32 tl = (u32)P << 1, th = (u32)(P >> 32) << 1;
+  const u32 sl = (u32)M + tl, sh_ = (u32)(M >> 32) + th;
+#else
   const u32 two = c_pow2[1];
   const u32 tl = (u32)P * two, th = (u32)(P >> 32) * two;
   const u32 sl = add_f((u32)M, tl), sh_ = add_f((u32)(M >> 32), th);
+#endif
   return join32(sl & ~tl, sh_ & ~th);
 }
 
@@ -231,11 +266,15 @@ __device__ __forceinline__ u64 east_moves_f(u64 P, u64 M) {
 // the other three axes by the doubled-propagator fill.
 __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
   const u64 M = O & kInner;
+#if MCTS_MG_EAST_CARRY
   u64 m = east_moves_f(P, M);
-  m |= axis_moves<8, kFma, kFma>(P, O);
-  m |= axis_moves<7, kFma, kFma>(P, M);
-  m |= axis_moves<9, kFma, kFma>(P, M);
   m |= __brevll(east_moves_f(rP, rO & kInner));
+#else
+  u64 m = axis_moves<1, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, M);
+#endif
+  m |= axis_moves<8, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, O);
+  m |= axis_moves<7, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, M);
+  m |= axis_moves<9, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, M);
   return m & ~(P | O);
 }
 
@@ -335,6 +374,16 @@ struct PlayoutRng {
   u32 w;
   uint4 buf;  // the unread words of the current Philox block, in order
   __device__ __forceinline__ u32 next() {
+#if MCTS_RNG_SELECT
+    const u32 lane = w & 3u;
+    if (lane == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
+    ++w;
+    u32 r = buf.x;
+    r = lane == 1u ? buf.y : r;
+    r = lane == 2u ? buf.z : r;
+    r = lane == 3u ? buf.w : r;
+    return r;
+#else
     if ((w & 3u) == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
     ++w;
     const u32 r = buf.x;
@@ -342,6 +391,7 @@ struct PlayoutRng {
     buf.y = buf.z;
     buf.z = buf.w;
     return r;
+#endif
   }
 };
 
@@ -365,10 +415,19 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
     } else {
       passed = false;
       const u32 r = rng.next();
+#if MCTS_PICK_F
       const int sq = kth_set_bit_f(moves, __umulhi(r, (u32)__popcll(moves)));
+#else
+      const int sq = kth_set_bit(moves, __umulhi(r, (u32)__popcll(moves)));
+#endif
       const u64 f = flips_hot(sq, me, op, rme, rop, rays);
+#if MCTS_UPD_F
       me = or_disjoint_f(me, or_disjoint_f(f, 1ULL << sq));
       op = andnot_subset_f(op, f);
+#else
+      me |= f | (1ULL << sq);
+      op &= ~f;
+#endif
       ++n;
     }
     const u64 t = me; me = op; op = t;
