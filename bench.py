@@ -146,6 +146,8 @@ def main():
     ap.add_argument("--no-search", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--search-ms", type=float, default=SEARCH_MS)
+    ap.add_argument("--search-iters", type=int, default=0,
+                    help="iteration-mode search legs (profiling); default: time mode")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -243,30 +245,37 @@ def main():
     e2e_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_s
 
     log('# ---- block-parallel search')
-    # ---- block-parallel search, configs[2] shape, time mode, + root allreduce
+    # ---- block-parallel search (configs[2] shape) and leaf-parallel comparison
+    # (configs[3]), time mode (or --search-iters for profiling), + root allreduce
     search = None
     leaf_search = None
     launches = args.steps  # one playouts_kernel per timed step
-    if not args.no_search:
+
+    def run_search(handle, n_trees, threads, id_base):
         root = pkg.position(*pkg.OPENING)
-        sstats = torch.zeros(198, dtype=torch.int64, device="cuda")
-        m.search_async(root, 0, 50.0, SEARCH_TREES, SEARCH_THREADS, 1000, rank * SEARCH_TREES,
-                       sstats.data_ptr(), stream)  # warm-up (pool + ln table)
+        st = torch.zeros(198, dtype=torch.int64, device="cuda")
+        it, ms = (args.search_iters, 0.0) if args.search_iters else (0, args.search_ms)
+        handle.search_async(root, min(it, 2) if it else 0, 0.0 if it else 20.0, n_trees, threads,
+                            1000, id_base, st.data_ptr(), stream)  # warm-up: pool + ln table
         torch.cuda.synchronize()
         barrier()
-        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s0.record(stream)
-        m.search_async(root, 0, args.search_ms, SEARCH_TREES, SEARCH_THREADS, 1000,
-                       rank * SEARCH_TREES, sstats.data_ptr(), stream)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        handle.search_async(root, it, ms, n_trees, threads, 1000, id_base, st.data_ptr(), stream)
         with torch.cuda.stream(stream):
-            merge_root_stats(sstats)
-        s1.record(stream)
+            merge_root_stats(st)  # the single cross-GPU collective (no-op at N=1)
+        e1.record(stream)
         torch.cuda.synchronize()
-        s_ms = max_over_ranks(s0.elapsed_time(s1))
-        st = sstats.cpu().numpy()
+        t_ms = max_over_ranks(e0.elapsed_time(e1))
+        return st.cpu().numpy(), t_ms
+
+    if not args.no_search:
+        mode = (f"{args.search_iters} iterations" if args.search_iters else
+                f"{args.search_ms:.0f} ms time mode")
+        st, s_ms = run_search(m, SEARCH_TREES, SEARCH_THREADS, rank * SEARCH_TREES)
         search = {
             "workload": f"configs[2] shape: {SEARCH_TREES} trees x {SEARCH_THREADS} threads per GPU, "
-                        f"{args.search_ms:.0f} ms time mode, opening root, C=1.0",
+                        f"{mode}, opening root, C=1.0",
             "playouts_per_s": float(st[195]) / (s_ms / 1e3), "ms": s_ms,
             "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
@@ -274,22 +283,12 @@ def main():
         }
         log('ml = pkg.Mcts(')
         ml = pkg.Mcts(c_uct=1.0, scheme="leaf", device=local)
-        lstats = torch.zeros(198, dtype=torch.int64, device="cuda")
-        ml.search_async(root, 0, 20.0, 1, LEAF_THREADS, 1000, rank, lstats.data_ptr(), stream)
-        torch.cuda.synchronize()
-        s0.record(stream)
-        ml.search_async(root, 0, args.search_ms, 1, LEAF_THREADS, 1000, rank, lstats.data_ptr(), stream)
-        with torch.cuda.stream(stream):
-            merge_root_stats(lstats)
-        s1.record(stream)
-        torch.cuda.synchronize()
-        l_ms = max_over_ranks(s0.elapsed_time(s1))
-        lt = lstats.cpu().numpy()
+        lt, l_ms = run_search(ml, 1, LEAF_THREADS, rank)
         leaf_search = {
-            "workload": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch per GPU, "
-                        f"{args.search_ms:.0f} ms",
+            "workload": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch per GPU, {mode}",
             "playouts_per_s": float(lt[195]) / (l_ms / 1e3), "ms": l_ms,
-            "iterations": float(lt[196]) / world, "best_move": int(pkg.best_move(lt)),
+            "iterations": float(lt[196]) / world, "plies_per_s": float(lt[197]) / (l_ms / 1e3),
+            "best_move": int(pkg.best_move(lt)),
         }
         ml.close()
 
@@ -312,9 +311,9 @@ def main():
     plies_per_launch = plies_local / args.steps
     achieved = plies_per_launch * ALG_OPS_PER_PLY / kern_s
     traffic = None
-    try:
+    try:  # DRAM bytes per launch of this kernel from the committed ncu --set full capture
         prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))
-        traffic = prof.get("dram_bytes_per_launch")
+        traffic = prof["playouts"]["dram_bytes_per_launch"]
     except Exception:
         pass
     line = {

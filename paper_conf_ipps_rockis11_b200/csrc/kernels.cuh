@@ -41,7 +41,7 @@ __device__ __forceinline__ u64 globaltimer_ns() {
 // and added with one atomic per counter; plies with one atomic per warp.
 // ---------------------------------------------------------------------------
 #ifndef MCTS_PLAYOUT_THREADS
-#define MCTS_PLAYOUT_THREADS 128
+#define MCTS_PLAYOUT_THREADS 256
 #endif
 #ifndef MCTS_PLAYOUT_MINB
 #define MCTS_PLAYOUT_MINB 1

@@ -116,6 +116,9 @@ enum { kAlu = 0, kFma = 1, kMix = 2 };
 #ifndef MCTS_FLIP_ADD_F
 #define MCTS_FLIP_ADD_F 0
 #endif
+#ifndef MCTS_MG_REVERSED
+#define MCTS_MG_REVERSED 1
+#endif
 #ifndef MCTS_RNG_SELECT
 #define MCTS_RNG_SELECT 0
 #endif
@@ -261,10 +264,37 @@ __device__ __forceinline__ u64 east_moves_f(u64 P, u64 M) {
   return join32(sl & ~tl, sh_ & ~th);
 }
 
-// Legal moves with the horizontal axis done by carries (west as east of the
-// bit-reversed board rP/rO, which the caller also reuses for the flips) and
-// the other three axes by the doubled-propagator fill.
+// One upward direction (+S, S in {7, 8, 9}) of the doubled-propagator fill,
+// left shifts only (lo: IMAD.SHL on the FMA pipe, hi: one funnel SHF).
+template <int S>
+__device__ __forceinline__ u64 up_moves(u64 P, u64 M) {
+  const u64 M2 = M & shl<S, kAlu>(M);
+  u64 t = M & shl<S, kAlu>(P);
+  t |= M & shl<S, kAlu>(t);
+  t |= M2 & shl<2 * S, kAlu>(t);
+  t |= M2 & shl<2 * S, kAlu>(t);
+  return shl<S, kAlu>(t);
+}
+
+// Legal moves. The four upward directions (+1 by carries, +7/+8/+9 by fills)
+// run on the board; the four downward ones run as upward directions of the
+// bit-reversed board rP/rO (square s -> 63 - s is the 180-degree rotation, so
+// -1/-7/-8/-9 become +1/+7/+8/+9 and the file masks are unchanged). Only left
+// shifts remain, which split evenly between the ALU and FMA pipes; the caller
+// reuses rP/rO for the flips.
 __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
+#if MCTS_MG_REVERSED
+  const u64 M = O & kInner, rM = rO & kInner;
+  u64 m = east_moves_f(P, M);
+  m |= up_moves<8>(P, O);
+  m |= up_moves<7>(P, M);
+  m |= up_moves<9>(P, M);
+  u64 r = east_moves_f(rP, rM);
+  r |= up_moves<8>(rP, rO);
+  r |= up_moves<7>(rP, rM);
+  r |= up_moves<9>(rP, rM);
+  return (m | __brevll(r)) & ~(P | O);
+#else
   const u64 M = O & kInner;
 #if MCTS_MG_EAST_CARRY
   u64 m = east_moves_f(P, M);
@@ -276,6 +306,7 @@ __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
   m |= axis_moves<7, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, M);
   m |= axis_moves<9, MCTS_MG_LEFT, MCTS_MG_RIGHT>(P, M);
   return m & ~(P | O);
+#endif
 }
 
 // flips_fast with the bit-reversed board supplied by the caller.

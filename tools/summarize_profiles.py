@@ -1,0 +1,64 @@
+"""Summaries of the round's ncu captures into profiles/ (committed evidence).
+usage: python tools/summarize_profiles.py TAG"""
+import csv, json, os, subprocess, sys
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ncu_summary import summary
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
+out_dir = os.path.join(ROOT, "profiles")
+os.makedirs(out_dir, exist_ok=True)
+latest = {}
+for k in ["playouts", "block_search"]:
+    rep = os.path.join(ROOT, "gpurun_out", f"{tag}_{k}.ncu-rep")
+    if not os.path.exists(rep):
+        continue
+    d = summary(rep)
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(raw.splitlines()))
+    h, u, v = rows[0], rows[1], rows[2]
+    extra = {}
+    for name in ["sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
+                 "sm__issue_active.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
+                 "smsp__thread_inst_executed.sum", "launch__grid_size", "launch__block_size"]:
+        if name in h:
+            extra[name] = (v[h.index(name)], u[h.index(name)])
+    d.update(extra)
+    with open(os.path.join(out_dir, f"{tag}_ncu_{k}.txt"), "w") as f:
+        f.write(f"# ncu --set full --clock-control none summary, kernel {k}, round tag {tag}\n")
+        for name, (val, unit) in d.items():
+            f.write(f"{name:80s} {val:>18s} {unit}\n")
+    def num(name):
+        val, unit = d[name]
+        x = float(val.replace(",", ""))
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+        return x * scale
+    latest[k] = {"dram_bytes_per_launch": num("dram__bytes_read.sum") + num("dram__bytes_write.sum"),
+                 "duration_us": num("gpu__time_duration.sum"),
+                 "thread_inst": float(d["smsp__inst_executed.sum"][0].replace(",", "")) *
+                 float(d["smsp__thread_inst_executed_per_inst_executed.ratio"][0])}
+launch_csv = os.path.join(ROOT, "gpurun_out", f"{tag}_launches.csv")
+if os.path.exists(launch_csv):
+    lines = open(launch_csv).read().splitlines()
+    start = next(i for i, l in enumerate(lines) if l.startswith('"ID"'))
+    rows = list(csv.reader(lines[start:]))
+    h = rows[0]
+    ki, vi = h.index("Kernel Name"), h.index("Metric Value")
+    tot = {}
+    for r in rows[1:]:
+        if len(r) <= vi:
+            continue
+        name = r[ki].split("(")[0]
+        tot.setdefault(name, [0, 0.0])
+        tot[name][0] += 1
+        tot[name][1] += float(r[vi].replace(",", ""))
+    with open(os.path.join(out_dir, f"{tag}_launches.txt"), "w") as f:
+        f.write("# ncu --metrics gpu__time_duration.sum --clock-control none, bench.py --steps 5 --warmup 3\n")
+        f.write("# (cold-cache serialised launches: compare shares, not absolutes)\n")
+        allt = sum(t for _, t in tot.values())
+        for name, (n, t) in sorted(tot.items(), key=lambda kv: -kv[1][1]):
+            f.write(f"{name:60s} launches {n:5d}  total {t/1e3:12.1f} us  share {100*t/allt:5.1f}%\n")
+    import shutil
+    shutil.copy(launch_csv, os.path.join(out_dir, f"{tag}_launches.csv"))
+json.dump(latest, open(os.path.join(out_dir, "latest_ncu.json"), "w"), indent=1)
+print(json.dumps(latest, indent=1))
