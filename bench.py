@@ -129,6 +129,112 @@ def cpu_baseline(budget_s=12.0):
             "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)"}
 
 
+def selfplay_leg(args, world, rank, local):
+    """Win% of the B200 searcher vs the multi-threaded CPU oracle MCTS at equal
+    wall time per move (BASELINE.json metric, configs[2]-[4]). Rank 0 referees
+    with the oracle's rules and plays the CPU side on all host cores; every rank
+    searches its own trees (tree_id_base = rank * n_trees) and the root stats
+    are merged by one allreduce per move, so all ranks agree on the move."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_rockis11_b200 as pkg
+    from paper_conf_ipps_rockis11_b200.distributed import merge_root_stats, best_move_from
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    scheme = args.sp_scheme
+    n_trees, threads = (SEARCH_TREES, SEARCH_THREADS) if scheme == "block" else (1, LEAF_THREADS)
+    m = pkg.Mcts(c_uct=1.0, scheme=scheme, device=local)
+    stream = torch.cuda.current_stream()
+    stats = torch.zeros(198, dtype=torch.int64, device="cuda")
+    msg = torch.zeros(4, dtype=torch.int64, device="cuda")  # black, white, to_move, seed/-1
+
+    def gpu_move(black, white, to_move, seed):
+        pos = pkg.position(black, white, to_move)
+        m.search_async(pos, 0, args.move_ms, n_trees, threads, seed, rank * n_trees,
+                       stats.data_ptr(), stream)
+        with torch.cuda.stream(stream):
+            merge_root_stats(stats)
+        torch.cuda.synchronize()
+        st = stats.cpu().numpy()
+        return best_move_from(st), int(st[195])
+
+    if rank != 0:  # follower ranks: search whatever position rank 0 broadcasts
+        while True:
+            dist.broadcast(msg, 0)
+            b, w, t, seed = (int(x) for x in msg.cpu().numpy())
+            if seed < 0:
+                break
+            gpu_move(b & ((1 << 64) - 1), w & ((1 << 64) - 1), t, seed)
+        dist.destroy_process_group()
+        return
+
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    def to_i64(x):
+        return x - (1 << 64) if x >= (1 << 63) else x
+    res = {"W": 0, "D": 0, "L": 0}
+    diffs, gpu_po, cpu_po = [], [], []
+    t_start = time.time()
+    for g in range(args.selfplay):
+        gpu_color = g % 2
+        black, white, to_move = oracle.OPENING_BLACK, oracle.OPENING_WHITE, 0
+        ply = 0
+        while True:
+            own, opp = (black, white) if to_move == 0 else (white, black)
+            legal = oracle.legal(own, opp)
+            if legal == 0:
+                if oracle.legal(opp, own) == 0:
+                    break
+                to_move ^= 1
+                continue
+            seed = 1000 + 1000 * g + ply
+            if to_move == gpu_color:
+                if world > 1:
+                    msg.copy_(torch.tensor([to_i64(black), to_i64(white), to_move, seed]))
+                    dist.broadcast(msg, 0)
+                mv, po = gpu_move(black, white, to_move, seed)
+                gpu_po.append(po)
+            else:
+                st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cores, args.move_ms, seed)
+                cpu_po.append(int(st[195]))
+            assert 0 <= mv < 64 and (legal >> mv) & 1, (mv, hex(legal))
+            f = oracle.flips(own, opp, mv)
+            own, opp = own | f | (1 << mv), opp & ~f
+            black, white = (own, opp) if to_move == 0 else (opp, own)
+            to_move ^= 1
+            ply += 1
+        gb = bin(black).count("1"), bin(white).count("1")
+        d = (gb[0] - gb[1]) if gpu_color == 0 else (gb[1] - gb[0])
+        diffs.append(d)
+        res["W" if d > 0 else "D" if d == 0 else "L"] += 1
+        log(f"game {g}: gpu={'black' if gpu_color == 0 else 'white'} diff {d:+d} {res}")
+    if world > 1:
+        msg.copy_(torch.tensor([0, 0, 0, -1]))
+        dist.broadcast(msg, 0)
+    n = max(args.selfplay, 1)
+    p = (res["W"] + 0.5 * res["D"]) / n
+    z = 1.96  # Wilson score interval
+    centre = (p + z * z / (2 * n)) / (1 + z * z / n)
+    half = z * float(np.sqrt(p * (1 - p) / n + z * z / (4 * n * n))) / (1 + z * z / n)
+    print(json.dumps({
+        "metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": 100 * p, "unit": "%",
+        "ci95_wilson": [100 * (centre - half), 100 * (centre + half)], "games": args.selfplay, "results": res, "n_gpus": world,
+        "mean_disc_diff": float(np.mean(diffs)) if diffs else None,
+        "config": {"workload": f"configs[{2 if scheme == 'block' else 3}] searcher "
+                               f"({n_trees} trees x {threads} threads per GPU, {scheme}) vs root-parallel "
+                               f"CPU oracle MCTS on {cores} host threads",
+                   "move_ms": args.move_ms, "colours": "alternating", "C": 1.0},
+        "gpu_playouts_per_move": float(np.mean(gpu_po)) if gpu_po else None,
+        "cpu_playouts_per_move": float(np.mean(cpu_po)) if cpu_po else None,
+        "wall_s": time.time() - t_start,
+    }), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def log(*a):
     if os.environ.get("BENCH_DEBUG"):
         print("[bench]", *a, file=sys.stderr, flush=True)
@@ -146,6 +252,10 @@ def main():
     ap.add_argument("--no-search", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--search-ms", type=float, default=SEARCH_MS)
+    ap.add_argument("--selfplay", type=int, default=0,
+                    help="play N games vs the CPU oracle MCTS and print the win%% line instead")
+    ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
+    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
     ap.add_argument("--search-iters", type=int, default=0,
                     help="iteration-mode search legs (profiling); default: time mode")
     args = ap.parse_args()
@@ -155,6 +265,8 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         return reference_arm(args, rank)
+    if args.selfplay:
+        return selfplay_leg(args, world, rank, local)
     if args.warmup < 3:
         args.warmup = 3
 
