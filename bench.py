@@ -129,6 +129,42 @@ def cpu_baseline(budget_s=12.0):
             "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)"}
 
 
+def sweep_leg(args, local):
+    """Fig. 5 analog (NEXT-2): search playouts/s vs total GPU
+    threads for leaf parallelism and block parallelism with 32- and 128-thread
+    blocks, time mode from the opening. One JSON line per point, rank 0 only."""
+    import torch
+    import paper_conf_ipps_rockis11_b200 as pkg
+    torch.cuda.set_device(local)
+    stream = torch.cuda.current_stream()
+    root = pkg.position(*pkg.OPENING)
+    st = torch.zeros(198, dtype=torch.int64, device="cuda")
+    handles = {"block": pkg.Mcts(scheme="block", device=local), "leaf": pkg.Mcts(scheme="leaf", device=local)}
+    points = []
+    for total in [128, 512, 2048, 8192, 16384, 37888, 75776, 151552]:
+        for scheme, bs in [("leaf", 128), ("block", 32), ("block", 128)]:
+            if scheme == "leaf" and total > 65536:
+                continue
+            n_trees, threads = (1, total) if scheme == "leaf" else (total // bs, bs)
+            h = handles[scheme]
+            h.search_async(root, 0, 10.0, n_trees, threads, 7, 0, st.data_ptr(), stream)  # warm-up
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            h.search_async(root, 0, args.sweep_ms, n_trees, threads, 7, 0, st.data_ptr(), stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1)
+            s = st.cpu().numpy()
+            points.append({"scheme": scheme, "block": bs, "gpu_threads": total, "trees": n_trees,
+                           "playouts_per_s": float(s[195]) / (ms / 1e3),
+                           "iterations_per_tree": float(s[196]) / n_trees, "ms": ms})
+            log(points[-1])
+    print(json.dumps({"metric": "search playouts/s vs GPU threads (Fig. 5 analog)", "unit": "playouts/s",
+                      "config": {"root": "opening", "time_ms": args.sweep_ms, "C": 1.0},
+                      "points": points}), flush=True)
+
+
 def selfplay_leg(args, world, rank, local):
     """Win% of the B200 searcher vs the multi-threaded CPU oracle MCTS at equal
     wall time per move (BASELINE.json metric, configs[2]-[4]). Rank 0 referees
@@ -256,6 +292,8 @@ def main():
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
     ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
+    ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
+    ap.add_argument("--sweep-ms", type=float, default=200.0)
     ap.add_argument("--search-iters", type=int, default=0,
                     help="iteration-mode search legs (profiling); default: time mode")
     args = ap.parse_args()
@@ -267,6 +305,8 @@ def main():
         return reference_arm(args, rank)
     if args.selfplay:
         return selfplay_leg(args, world, rank, local)
+    if args.sweep:
+        return sweep_leg(args, local) if rank == 0 else None
     if args.warmup < 3:
         args.warmup = 3
 

@@ -119,6 +119,28 @@ enum { kAlu = 0, kFma = 1, kMix = 2 };
 #ifndef MCTS_MG_REVERSED
 #define MCTS_MG_REVERSED 1
 #endif
+// per-step shift pipe of up_moves (kAlu: IMAD.SHL + funnel SHF; kFma: IMAD.WIDE + IMAD)
+#ifndef MCTS_UP_M2
+#define MCTS_UP_M2 kAlu
+#endif
+#ifndef MCTS_UP_S1
+#define MCTS_UP_S1 kAlu
+#endif
+#ifndef MCTS_UP_S2
+#define MCTS_UP_S2 kAlu
+#endif
+#ifndef MCTS_UP_D1
+#define MCTS_UP_D1 kAlu
+#endif
+#ifndef MCTS_UP_D2
+#define MCTS_UP_D2 kAlu
+#endif
+#ifndef MCTS_UP_FIN
+#define MCTS_UP_FIN kAlu
+#endif
+#ifndef MCTS_PICK_LUT
+#define MCTS_PICK_LUT 0
+#endif
 #ifndef MCTS_RNG_SELECT
 #define MCTS_RNG_SELECT 0
 #endif
@@ -194,7 +216,9 @@ __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
   return m;
 }
 
-constexpr int kRayTable = 512;
+// Shared per-CTA table: [0,256) ray masks, [256,512) first ray squares,
+// [512,768) a byte-select LUT: byte (k*256 + b) = index of the k-th set bit of b.
+constexpr int kRayTable = 768;
 
 // Flips along an upward ray by carry propagation: adding the ray's first square
 // to (O | ~m) carries through the contiguous opponent run (and through the
@@ -268,12 +292,12 @@ __device__ __forceinline__ u64 east_moves_f(u64 P, u64 M) {
 // left shifts only (lo: IMAD.SHL on the FMA pipe, hi: one funnel SHF).
 template <int S>
 __device__ __forceinline__ u64 up_moves(u64 P, u64 M) {
-  const u64 M2 = M & shl<S, kAlu>(M);
-  u64 t = M & shl<S, kAlu>(P);
-  t |= M & shl<S, kAlu>(t);
-  t |= M2 & shl<2 * S, kAlu>(t);
-  t |= M2 & shl<2 * S, kAlu>(t);
-  return shl<S, kAlu>(t);
+  const u64 M2 = M & shl<S, MCTS_UP_M2>(M);
+  u64 t = M & shl<S, MCTS_UP_S1>(P);
+  t |= M & shl<S, MCTS_UP_S2>(t);
+  t |= M2 & shl<2 * S, MCTS_UP_D1>(t);
+  t |= M2 & shl<2 * S, MCTS_UP_D2>(t);
+  return shl<S, MCTS_UP_FIN>(t);
 }
 
 // Legal moves. The four upward directions (+1 by carries, +7/+8/+9 by fills)
@@ -377,6 +401,19 @@ __device__ __forceinline__ int kth_set_bit(u64 m, u32 k) {
   return base;
 }
 
+// k-th set bit: three popc levels down to a byte, then the byte-select LUT.
+__device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char* __restrict__ lut) {
+  u32 lo = (u32)m, hi = (u32)(m >> 32);
+  u32 c = __popc(lo);
+  bool up = k >= c;
+  u32 x = up ? hi : lo;
+  k -= up ? c : 0u;
+  int base = up ? 32 : 0;
+  c = __popc(x & 0xFFFFu); up = k >= c; x = up ? (x >> 16) : x; k -= up ? c : 0u; base += up ? 16 : 0;
+  c = __popc(x & 0xFFu);   up = k >= c; x = up ? (x >> 8) : x;  k -= up ? c : 0u; base += up ? 8 : 0;
+  return base + lut[(k << 8) | (x & 0xFFu)];
+}
+
 // Uniform pick (R4): k = floor(r * c / 2^32), then the k-th legal
 // square in ascending order.
 __device__ __forceinline__ int pick_square(u64 moves, u32 r) {
@@ -448,6 +485,9 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
       const u32 r = rng.next();
 #if MCTS_PICK_F
       const int sq = kth_set_bit_f(moves, __umulhi(r, (u32)__popcll(moves)));
+#elif MCTS_PICK_LUT
+      const int sq = kth_set_bit_lut(moves, __umulhi(r, (u32)__popcll(moves)),
+                                     reinterpret_cast<const unsigned char*>(rays + 512));
 #else
       const int sq = kth_set_bit(moves, __umulhi(r, (u32)__popcll(moves)));
 #endif
@@ -476,6 +516,15 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
     const u64 m = ray_mask(i >> 6, i & 63);
     rays[i] = m;
     rays[256 + i] = m & (0ULL - m);  // lowest ray square (0 if the ray is empty)
+    u64 packed = 0;                  // LUT bytes 8i .. 8i+7
+    for (int j = 0; j < 8; ++j) {
+      const int e = 8 * i + j, k = e >> 8, b = e & 255;
+      int seen = 0, pos = 0;
+      for (int q = 0; q < 8; ++q)
+        if ((b >> q) & 1) { if (seen == k) { pos = q; break; } ++seen; }
+      packed |= (u64)pos << (8 * j);
+    }
+    rays[512 + i] = packed;
   }
 }
 

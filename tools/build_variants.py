@@ -3,17 +3,20 @@ import os, sys, concurrent.futures as cf
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_rockis11_b200 import _build
 
+F = "kFma"
 VARIANTS = {
     "base": [],
-    "not_reversed": ["MCTS_MG_REVERSED=0"],
+    "up_all_fma": [f"MCTS_UP_M2={F}", f"MCTS_UP_S1={F}", f"MCTS_UP_S2={F}", f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}", f"MCTS_UP_FIN={F}"],
+    "up_m2_fin": [f"MCTS_UP_M2={F}", f"MCTS_UP_FIN={F}"],
+    "up_s1_s2": [f"MCTS_UP_S1={F}", f"MCTS_UP_S2={F}"],
+    "up_d1_d2": [f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}"],
+    "up_m2_s1_d1": [f"MCTS_UP_M2={F}", f"MCTS_UP_S1={F}", f"MCTS_UP_D1={F}"],
+    "up_s1_d1_fin": [f"MCTS_UP_S1={F}", f"MCTS_UP_D1={F}", f"MCTS_UP_FIN={F}"],
+    "up_m2": [f"MCTS_UP_M2={F}"],
+    "up_fin": [f"MCTS_UP_FIN={F}"],
     "upd_f": ["MCTS_UPD_F=1"],
-    "flipadd_f": ["MCTS_FLIP_ADD_F=1"],
-    "upd_flipadd_f": ["MCTS_UPD_F=1", "MCTS_FLIP_ADD_F=1"],
-    "east_plain": ["MCTS_EAST_PLAIN=1"],
-    "t256": ["MCTS_PLAYOUT_THREADS=256"],
-    "minb8": ["MCTS_PLAYOUT_MINB=8"],
-    "minb9": ["MCTS_PLAYOUT_MINB=9"],
-    "upd_f_t256": ["MCTS_UPD_F=1", "MCTS_PLAYOUT_THREADS=256"],
+    "pick_lut": ["MCTS_PICK_LUT=1"],
+    "pick_lut_up_d1_d2": ["MCTS_PICK_LUT=1", f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}"],
 }
 
 if __name__ == "__main__":
