@@ -111,7 +111,7 @@ enum { kAlu = 0, kFma = 1, kMix = 2 };
 #define MCTS_PICK_F 0
 #endif
 #ifndef MCTS_UPD_F
-#define MCTS_UPD_F 0
+#define MCTS_UPD_F 1
 #endif
 #ifndef MCTS_FLIP_ADD_F
 #define MCTS_FLIP_ADD_F 0
@@ -139,7 +139,7 @@ enum { kAlu = 0, kFma = 1, kMix = 2 };
 #define MCTS_UP_FIN kAlu
 #endif
 #ifndef MCTS_PICK_LUT
-#define MCTS_PICK_LUT 0
+#define MCTS_PICK_LUT 1
 #endif
 #ifndef MCTS_RNG_SELECT
 #define MCTS_RNG_SELECT 0
@@ -463,49 +463,53 @@ struct PlayoutRng {
   }
 };
 
+// One decision for the side owning P: returns false if P has no move (a pass;
+// nothing changes), else plays the random move and returns true.
+__device__ __forceinline__ bool ply(u64& P, u64& O, PlayoutRng& rng, const u64* __restrict__ rays) {
+  const u64 rP = __brevll(P), rO = __brevll(O);
+  const u64 moves = legal_moves_hot(P, O, rP, rO);
+  if (moves == 0ULL) return false;
+  const u32 r = rng.next();
+#if MCTS_PICK_F
+  const int sq = kth_set_bit_f(moves, __umulhi(r, (u32)__popcll(moves)));
+#elif MCTS_PICK_LUT
+  const int sq = kth_set_bit_lut(moves, __umulhi(r, (u32)__popcll(moves)),
+                                 reinterpret_cast<const unsigned char*>(rays + 512));
+#else
+  const int sq = kth_set_bit(moves, __umulhi(r, (u32)__popcll(moves)));
+#endif
+  const u64 f = flips_hot(sq, P, O, rP, rO, rays);
+#if MCTS_UPD_F
+  P = or_disjoint_f(P, or_disjoint_f(f, 1ULL << sq));
+  O = andnot_subset_f(O, f);
+#else
+  P |= f | (1ULL << sq);
+  O &= ~f;
+#endif
+  return true;
+}
+
 // One random playout from (me to move, op). Returns +1 / 0 / -1 for the side
 // to move at the start (R3), adds the non-pass plies to *plies.
-// A pass consumes no RNG word; two consecutive passes end the game.
+// A pass consumes no RNG word; two consecutive passes end the game. The loop is
+// unrolled by two so the sides keep their registers (no swaps).
 __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1, u32 c2,
                                        const u64* __restrict__ rays, u32* plies) {
   PlayoutRng rng;
   rng.key = key; rng.c0 = c0; rng.c1 = c1; rng.c2 = c2; rng.w = 0;
   rng.buf = make_uint4(0, 0, 0, 0);
-  bool start = true;   // does `me` belong to the player who was to move at the start?
   bool passed = false;
   u32 n = 0;
   for (;;) {
-    const u64 rme = __brevll(me), rop = __brevll(op);
-    const u64 moves = legal_moves_hot(me, op, rme, rop);
-    if (moves == 0ULL) {
-      if (passed) break;  // neither player can move
-      passed = true;
-    } else {
-      passed = false;
-      const u32 r = rng.next();
-#if MCTS_PICK_F
-      const int sq = kth_set_bit_f(moves, __umulhi(r, (u32)__popcll(moves)));
-#elif MCTS_PICK_LUT
-      const int sq = kth_set_bit_lut(moves, __umulhi(r, (u32)__popcll(moves)),
-                                     reinterpret_cast<const unsigned char*>(rays + 512));
-#else
-      const int sq = kth_set_bit(moves, __umulhi(r, (u32)__popcll(moves)));
-#endif
-      const u64 f = flips_hot(sq, me, op, rme, rop, rays);
-#if MCTS_UPD_F
-      me = or_disjoint_f(me, or_disjoint_f(f, 1ULL << sq));
-      op = andnot_subset_f(op, f);
-#else
-      me |= f | (1ULL << sq);
-      op &= ~f;
-#endif
-      ++n;
-    }
-    const u64 t = me; me = op; op = t;
-    start = !start;
+    if (ply(me, op, rng, rays)) { passed = false; ++n; }
+    else if (passed) break;  // neither player can move
+    else passed = true;
+    if (ply(op, me, rng, rays)) { passed = false; ++n; }
+    else if (passed) break;
+    else passed = true;
   }
   *plies += n;
-  const int a = __popcll(start ? me : op), b = __popcll(start ? op : me);
+  const int a = __popcll(me), b = __popcll(op);
   return (a > b) - (a < b);
 }
 

@@ -6,17 +6,11 @@ from paper_conf_ipps_rockis11_b200 import _build
 F = "kFma"
 VARIANTS = {
     "base": [],
-    "up_all_fma": [f"MCTS_UP_M2={F}", f"MCTS_UP_S1={F}", f"MCTS_UP_S2={F}", f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}", f"MCTS_UP_FIN={F}"],
-    "up_m2_fin": [f"MCTS_UP_M2={F}", f"MCTS_UP_FIN={F}"],
-    "up_s1_s2": [f"MCTS_UP_S1={F}", f"MCTS_UP_S2={F}"],
-    "up_d1_d2": [f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}"],
-    "up_m2_s1_d1": [f"MCTS_UP_M2={F}", f"MCTS_UP_S1={F}", f"MCTS_UP_D1={F}"],
-    "up_s1_d1_fin": [f"MCTS_UP_S1={F}", f"MCTS_UP_D1={F}", f"MCTS_UP_FIN={F}"],
-    "up_m2": [f"MCTS_UP_M2={F}"],
-    "up_fin": [f"MCTS_UP_FIN={F}"],
+    "no_lut": ["MCTS_PICK_LUT=0"],
     "upd_f": ["MCTS_UPD_F=1"],
-    "pick_lut": ["MCTS_PICK_LUT=1"],
-    "pick_lut_up_d1_d2": ["MCTS_PICK_LUT=1", f"MCTS_UP_D1={F}", f"MCTS_UP_D2={F}"],
+    "t128": ["MCTS_PLAYOUT_THREADS=128"],
+    "minb4": ["MCTS_PLAYOUT_MINB=4"],
+    "minb3": ["MCTS_PLAYOUT_MINB=3"],
 }
 
 if __name__ == "__main__":
