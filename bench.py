@@ -159,10 +159,81 @@ def sweep_leg(args, local):
             points.append({"scheme": scheme, "block": bs, "gpu_threads": total, "trees": n_trees,
                            "playouts_per_s": float(s[195]) / (ms / 1e3),
                            "iterations_per_tree": float(s[196]) / n_trees, "ms": ms})
+            if args.sweep_games and total in (512, 2048, 16384, 151552):
+                def gpu_move(black, white, to_move, seed, h=h, n_trees=n_trees, threads=threads):
+                    h.search_async(pkg.position(black, white, to_move), 0, args.move_ms, n_trees, threads,
+                                   seed, 0, st.data_ptr(), stream)
+                    torch.cuda.synchronize()
+                    x = st.cpu().numpy()
+                    return pkg.best_move(x), int(x[195])
+                r = play_match(gpu_move, 1, args.sweep_games, args.move_ms, tag=f"{scheme}{bs}/{total}")
+                points[-1]["vs_1core"] = {k: r[k] for k in ("win_pct", "ci95_wilson", "results",
+                                                            "mean_disc_diff", "gpu_playouts_per_move",
+                                                            "cpu_playouts_per_move")}
             log(points[-1])
-    print(json.dumps({"metric": "search playouts/s vs GPU threads (Fig. 5 analog)", "unit": "playouts/s",
-                      "config": {"root": "opening", "time_ms": args.sweep_ms, "C": 1.0},
+    print(json.dumps({"metric": "search playouts/s vs GPU threads (Fig. 5 analog); win% vs 1 CPU core "
+                                "(Fig. 6 analog, points with vs_1core)", "unit": "playouts/s",
+                      "config": {"root": "opening", "time_ms": args.sweep_ms, "C": 1.0,
+                                 "games_per_point": args.sweep_games, "move_ms": args.move_ms},
                       "points": points}), flush=True)
+
+
+def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag=""):
+    """Games of the B200 searcher (gpu_move(black, white, to_move, seed) ->
+    (move, playouts)) against the oracle's root-parallel CPU MCTS on
+    `cpu_threads` host threads, alternating colours, equal time per move; the
+    oracle's rules referee. Returns W/D/L, disc differences and the per-game-step
+    disc difference (GPU minus CPU, the paper's "point difference")."""
+    import numpy as np
+    import oracle
+    res = {"W": 0, "D": 0, "L": 0}
+    diffs, gpu_po, cpu_po, steps = [], [], [], []
+    t_start = time.time()
+    for g in range(games):
+        gpu_color = g % 2
+        black, white, to_move = oracle.OPENING_BLACK, oracle.OPENING_WHITE, 0
+        ply, curve = 0, []
+        while True:
+            own, opp = (black, white) if to_move == 0 else (white, black)
+            legal = oracle.legal(own, opp)
+            if legal == 0:
+                if oracle.legal(opp, own) == 0:
+                    break
+                to_move ^= 1
+                continue
+            seed = seed_base + 1000 * g + ply
+            if to_move == gpu_color:
+                mv, po = gpu_move(black, white, to_move, seed)
+                gpu_po.append(po)
+            else:
+                st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cpu_threads, move_ms, seed)
+                cpu_po.append(int(st[195]))
+            assert 0 <= mv < 64 and (legal >> mv) & 1, (mv, hex(legal))
+            f = oracle.flips(own, opp, mv)
+            own, opp = own | f | (1 << mv), opp & ~f
+            black, white = (own, opp) if to_move == 0 else (opp, own)
+            to_move ^= 1
+            ply += 1
+            nb, nw = bin(black).count("1"), bin(white).count("1")
+            curve.append((nb - nw) if gpu_color == 0 else (nw - nb))
+        d = curve[-1] if curve else 0
+        diffs.append(d)
+        steps.append(curve)
+        res["W" if d > 0 else "D" if d == 0 else "L"] += 1
+        log(f"{tag} game {g}: gpu={'black' if gpu_color == 0 else 'white'} diff {d:+d} {res}")
+    n = max(games, 1)
+    p = (res["W"] + 0.5 * res["D"]) / n
+    z = 1.96  # Wilson score interval
+    centre = (p + z * z / (2 * n)) / (1 + z * z / n)
+    half = z * float(np.sqrt(p * (1 - p) / n + z * z / (4 * n * n))) / (1 + z * z / n)
+    L = max((len(c) for c in steps), default=0)
+    per_step = [float(np.mean([c[i] if i < len(c) else c[-1] for c in steps])) for i in range(L)]
+    return {"win_pct": 100 * p, "ci95_wilson": [100 * (centre - half), 100 * (centre + half)],
+            "results": res, "games": games, "mean_disc_diff": float(np.mean(diffs)) if diffs else None,
+            "point_diff_per_step": per_step,
+            "gpu_playouts_per_move": float(np.mean(gpu_po)) if gpu_po else None,
+            "cpu_playouts_per_move": float(np.mean(cpu_po)) if cpu_po else None,
+            "wall_s": time.time() - t_start}
 
 
 def selfplay_leg(args, world, rank, local):
@@ -170,8 +241,9 @@ def selfplay_leg(args, world, rank, local):
     wall time per move (BASELINE.json metric, configs[2]-[4]). Rank 0 referees
     with the oracle's rules and plays the CPU side on all host cores; every rank
     searches its own trees (tree_id_base = rank * n_trees) and the root stats
-    are merged by one allreduce per move, so all ranks agree on the move."""
-    import numpy as np
+    are merged by one allreduce per move, so all ranks agree on the move.
+    --fig7 instead sweeps the CPU side over 1, 2, 4, ... host threads and reports
+    the point difference per game step (Fig. 7 analog)."""
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_rockis11_b200 as pkg
@@ -187,7 +259,7 @@ def selfplay_leg(args, world, rank, local):
     stats = torch.zeros(198, dtype=torch.int64, device="cuda")
     msg = torch.zeros(4, dtype=torch.int64, device="cuda")  # black, white, to_move, seed/-1
 
-    def gpu_move(black, white, to_move, seed):
+    def search(black, white, to_move, seed):
         pos = pkg.position(black, white, to_move)
         m.search_async(pos, 0, args.move_ms, n_trees, threads, seed, rank * n_trees,
                        stats.data_ptr(), stream)
@@ -203,70 +275,43 @@ def selfplay_leg(args, world, rank, local):
             b, w, t, seed = (int(x) for x in msg.cpu().numpy())
             if seed < 0:
                 break
-            gpu_move(b & ((1 << 64) - 1), w & ((1 << 64) - 1), t, seed)
+            search(b & ((1 << 64) - 1), w & ((1 << 64) - 1), t, seed)
         dist.destroy_process_group()
         return
 
-    import oracle
-    cores = len(os.sched_getaffinity(0))
     def to_i64(x):
         return x - (1 << 64) if x >= (1 << 63) else x
-    res = {"W": 0, "D": 0, "L": 0}
-    diffs, gpu_po, cpu_po = [], [], []
-    t_start = time.time()
-    for g in range(args.selfplay):
-        gpu_color = g % 2
-        black, white, to_move = oracle.OPENING_BLACK, oracle.OPENING_WHITE, 0
-        ply = 0
-        while True:
-            own, opp = (black, white) if to_move == 0 else (white, black)
-            legal = oracle.legal(own, opp)
-            if legal == 0:
-                if oracle.legal(opp, own) == 0:
-                    break
-                to_move ^= 1
-                continue
-            seed = 1000 + 1000 * g + ply
-            if to_move == gpu_color:
-                if world > 1:
-                    msg.copy_(torch.tensor([to_i64(black), to_i64(white), to_move, seed]))
-                    dist.broadcast(msg, 0)
-                mv, po = gpu_move(black, white, to_move, seed)
-                gpu_po.append(po)
-            else:
-                st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cores, args.move_ms, seed)
-                cpu_po.append(int(st[195]))
-            assert 0 <= mv < 64 and (legal >> mv) & 1, (mv, hex(legal))
-            f = oracle.flips(own, opp, mv)
-            own, opp = own | f | (1 << mv), opp & ~f
-            black, white = (own, opp) if to_move == 0 else (opp, own)
-            to_move ^= 1
-            ply += 1
-        gb = bin(black).count("1"), bin(white).count("1")
-        d = (gb[0] - gb[1]) if gpu_color == 0 else (gb[1] - gb[0])
-        diffs.append(d)
-        res["W" if d > 0 else "D" if d == 0 else "L"] += 1
-        log(f"game {g}: gpu={'black' if gpu_color == 0 else 'white'} diff {d:+d} {res}")
+
+    def gpu_move(black, white, to_move, seed):
+        if world > 1:
+            msg.copy_(torch.tensor([to_i64(black), to_i64(white), to_move, seed]))
+            dist.broadcast(msg, 0)
+        return search(black, white, to_move, seed)
+
+    cores = len(os.sched_getaffinity(0))
+    workload = (f"configs[{2 if scheme == 'block' else 3}] searcher ({n_trees} trees x {threads} "
+                f"threads per GPU, {scheme}, {world} GPU(s))")
+    if args.fig7:
+        curves = []
+        t = 1
+        while t <= cores:
+            r = play_match(gpu_move, t, args.selfplay, args.move_ms, tag=f"cpu{t}")
+            curves.append({"cpu_threads": t, **r})
+            t *= 2
+        out = {"metric": "point difference per game step vs root-parallel CPU MCTS on 1..N host threads "
+                         "(Fig. 7 analog)", "unit": "discs", "n_gpus": world,
+               "config": {"workload": workload, "move_ms": args.move_ms, "games_per_point": args.selfplay,
+                          "C": 1.0}, "curves": curves}
+    else:
+        r = play_match(gpu_move, cores, args.selfplay, args.move_ms)
+        out = {"metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": r["win_pct"],
+               "unit": "%", "n_gpus": world,
+               "config": {"workload": workload + f" vs root-parallel CPU oracle MCTS on {cores} host threads",
+                          "move_ms": args.move_ms, "colours": "alternating", "C": 1.0}, **r}
     if world > 1:
         msg.copy_(torch.tensor([0, 0, 0, -1]))
         dist.broadcast(msg, 0)
-    n = max(args.selfplay, 1)
-    p = (res["W"] + 0.5 * res["D"]) / n
-    z = 1.96  # Wilson score interval
-    centre = (p + z * z / (2 * n)) / (1 + z * z / n)
-    half = z * float(np.sqrt(p * (1 - p) / n + z * z / (4 * n * n))) / (1 + z * z / n)
-    print(json.dumps({
-        "metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": 100 * p, "unit": "%",
-        "ci95_wilson": [100 * (centre - half), 100 * (centre + half)], "games": args.selfplay, "results": res, "n_gpus": world,
-        "mean_disc_diff": float(np.mean(diffs)) if diffs else None,
-        "config": {"workload": f"configs[{2 if scheme == 'block' else 3}] searcher "
-                               f"({n_trees} trees x {threads} threads per GPU, {scheme}) vs root-parallel "
-                               f"CPU oracle MCTS on {cores} host threads",
-                   "move_ms": args.move_ms, "colours": "alternating", "C": 1.0},
-        "gpu_playouts_per_move": float(np.mean(gpu_po)) if gpu_po else None,
-        "cpu_playouts_per_move": float(np.mean(cpu_po)) if cpu_po else None,
-        "wall_s": time.time() - t_start,
-    }), flush=True)
+    print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
 
@@ -292,7 +337,10 @@ def main():
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
     ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
+    ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
+    ap.add_argument("--sweep-games", type=int, default=0,
+                    help="with --sweep: also play N games per point vs 1-core CPU MCTS (Fig. 6 analog)")
     ap.add_argument("--sweep-ms", type=float, default=200.0)
     ap.add_argument("--search-iters", type=int, default=0,
                     help="iteration-mode search legs (profiling); default: time mode")
