@@ -1,16 +1,16 @@
-"""Build libmcts.so tuning variants into build/variants/ (see tools/variant_bench.cu)."""
+"""Build libmcts.so tuning variants into build/variants/ (see tools/variant_bench.cu).
+Knobs: MCTS_PICK_LUT, MCTS_UPD_F, MCTS_EAST_F (reversi_device.cuh),
+MCTS_PLAYOUT_THREADS, MCTS_PLAYOUT_MINB (kernels.cuh)."""
 import os, sys, concurrent.futures as cf
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_rockis11_b200 import _build
 
-F = "kFma"
 VARIANTS = {
     "base": [],
     "no_lut": ["MCTS_PICK_LUT=0"],
-    "upd_f": ["MCTS_UPD_F=1"],
+    "no_upd_f": ["MCTS_UPD_F=0"],
+    "no_east_f": ["MCTS_EAST_F=0"],
     "t128": ["MCTS_PLAYOUT_THREADS=128"],
-    "minb4": ["MCTS_PLAYOUT_MINB=4"],
-    "minb3": ["MCTS_PLAYOUT_MINB=3"],
 }
 
 if __name__ == "__main__":
