@@ -251,10 +251,10 @@ def selfplay_leg(args, world, rank, local):
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        init_dist(dist, torch, local)
     scheme = args.sp_scheme
     n_trees, threads = (SEARCH_TREES, SEARCH_THREADS) if scheme == "block" else (1, LEAF_THREADS)
-    m = pkg.Mcts(c_uct=1.0, scheme=scheme, device=local)
+    m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
     stream = torch.cuda.current_stream()
     stats = torch.zeros(198, dtype=torch.int64, device="cuda")
     msg = torch.zeros(4, dtype=torch.int64, device="cuda")  # black, white, to_move, seed/-1
@@ -301,19 +301,28 @@ def selfplay_leg(args, world, rank, local):
         out = {"metric": "point difference per game step vs root-parallel CPU MCTS on 1..N host threads "
                          "(Fig. 7 analog)", "unit": "discs", "n_gpus": world,
                "config": {"workload": workload, "move_ms": args.move_ms, "games_per_point": args.selfplay,
-                          "C": 1.0}, "curves": curves}
+                          "C": args.c_uct}, "curves": curves}
     else:
         r = play_match(gpu_move, cores, args.selfplay, args.move_ms)
         out = {"metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": r["win_pct"],
                "unit": "%", "n_gpus": world,
                "config": {"workload": workload + f" vs root-parallel CPU oracle MCTS on {cores} host threads",
-                          "move_ms": args.move_ms, "colours": "alternating", "C": 1.0}, **r}
+                          "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct}, **r}
     if world > 1:
         msg.copy_(torch.tensor([0, 0, 0, -1]))
         dist.broadcast(msg, 0)
     print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def init_dist(dist, torch, local):
+    """One process per GPU over NCCL (BENCH_BACKEND=gloo is a single-GPU test hook)."""
+    backend = os.environ.get("BENCH_BACKEND", "nccl")
+    if backend == "nccl":
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    else:
+        dist.init_process_group(backend)
 
 
 def log(*a):
@@ -337,6 +346,7 @@ def main():
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
     ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
+    ap.add_argument("--c-uct", type=float, default=1.0, help="UCB constant C of the GPU searcher")
     ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
     ap.add_argument("--sweep-games", type=int, default=0,
@@ -349,6 +359,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("BENCH_SAME_DEVICE"):  # test hook: all ranks on GPU 0 (with BENCH_BACKEND=gloo)
+        local = 0
     if args.impl == "reference":
         return reference_arm(args, rank)
     if args.selfplay:
@@ -367,7 +379,7 @@ def main():
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        init_dist(dist, torch, local)
 
     def barrier():
         if world > 1:
