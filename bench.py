@@ -522,10 +522,13 @@ def main():
     kern_s = kernel_ms / 1e3 / args.steps
     plies_per_launch = plies_local / args.steps
     achieved = plies_per_launch * ALG_OPS_PER_PLY / kern_s
-    traffic = None
-    try:  # DRAM bytes per launch of this kernel from the committed ncu --set full capture
-        prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))
-        traffic = prof["playouts"]["dram_bytes_per_launch"]
+    traffic, ncu = None, None
+    try:  # from the committed ncu --set full capture of this kernel (profiles/latest_ncu.json)
+        prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))["playouts"]
+        traffic = prof["dram_bytes_per_launch"]
+        ncu = {k: prof.get(k) for k in ("alu_pipe_pct", "fmaheavy_pipe_pct", "issue_active_pct",
+                                        "lanes_active_per_inst", "thread_inst")}
+        ncu["thread_inst_per_ply"] = prof["thread_inst"] / plies_per_launch if prof.get("thread_inst") else None
     except Exception:
         pass
     line = {
@@ -541,7 +544,7 @@ def main():
         "plies_per_s": plies_total / (t_ms / 1e3),
         "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak_ops / 1e9,
                      "unit": "Gop/s", "frac": achieved / peak_ops, "traffic": traffic,
-                     "ops_per_ply": ALG_OPS_PER_PLY, "plies_per_launch": plies_per_launch,
+                     "ops_per_ply": ALG_OPS_PER_PLY, "plies_per_launch": plies_per_launch, "ncu": ncu,
                      "peak_basis": f"issue slots 148 SM x 4 SMSP x 32 lanes x {sm_max:.0f} MHz "
                                    "(MEASURED_PEAKS.json sm_max_mhz), DESIGN.md §6"},
         "e2e": {"value": e2e_value, "unit": "playouts/s",

@@ -9,7 +9,7 @@ tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 out_dir = os.path.join(ROOT, "profiles")
 os.makedirs(out_dir, exist_ok=True)
 latest = {}
-for k in ["playouts", "block_search"]:
+for k in ["playouts", "block_search", "leaf_search"]:
     rep = os.path.join(ROOT, "gpurun_out", f"{tag}_{k}.ncu-rep")
     if not os.path.exists(rep):
         continue
@@ -33,7 +33,13 @@ for k in ["playouts", "block_search"]:
         x = float(val.replace(",", ""))
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
         return x * scale
-    latest[k] = {"dram_bytes_per_launch": num("dram__bytes_read.sum") + num("dram__bytes_write.sum"),
+    def pct(name):
+        return float(d[name][0]) if name in d else None
+    latest[k] = {"alu_pipe_pct": pct("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active"),
+                 "fmaheavy_pipe_pct": pct("sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+                 "issue_active_pct": pct("sm__issue_active.avg.pct_of_peak_sustained_elapsed"),
+                 "lanes_active_per_inst": pct("smsp__thread_inst_executed_per_inst_executed.ratio"),
+                 "dram_bytes_per_launch": num("dram__bytes_read.sum") + num("dram__bytes_write.sum"),
                  "duration_us": num("gpu__time_duration.sum"),
                  "thread_inst": float(d["smsp__inst_executed.sum"][0].replace(",", "")) *
                  float(d["smsp__thread_inst_executed_per_inst_executed.ratio"][0])}
