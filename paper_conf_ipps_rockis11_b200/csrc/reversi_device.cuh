@@ -349,10 +349,17 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   rng.buf = make_uint4(0, 0, 0, 0);
   bool passed = false;
   u32 n = 0;
+  // Every move fills one empty square, so the board is full (neither side can
+  // move: game over) exactly when n reaches the starting number of empties;
+  // testing that skips the two move generations that would establish it at the
+  // end of most random games.
+  const u32 empties = 64u - (u32)__popcll(me | op);
   for (;;) {
+    if (n == empties) break;
     if (ply(me, op, rng, rays)) { passed = false; ++n; }
     else if (passed) break;
     else passed = true;
+    if (n == empties) break;
     if (ply(op, me, rng, rays)) { passed = false; ++n; }
     else if (passed) break;
     else passed = true;
