@@ -492,6 +492,9 @@ def main():
             "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
+            # same per-ply op model as the headline roofline, per GPU
+            "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ALG_OPS_PER_PLY
+                             / (148 * 4 * 32 * measured_peaks().get("sm_max_mhz", 1965.0) * 1e6),
         }
         log('ml = pkg.Mcts(')
         ml = pkg.Mcts(c_uct=1.0, scheme="leaf", device=local)
