@@ -346,7 +346,9 @@ def main():
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
     ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
-    ap.add_argument("--c-uct", type=float, default=1.0, help="UCB constant C of the GPU searcher")
+    ap.add_argument("--c-uct", type=float, default=0.25,
+                    help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
+                         "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
     ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
     ap.add_argument("--sweep-games", type=int, default=0,

@@ -260,3 +260,41 @@ def test_search_invalid_arguments(mcts, orc):
     with pytest.raises(pkg.MctsError) as ei:
         mcts.search(orc.position(3, 1, 0), iterations=2, n_trees=1, threads_per_tree=32, seed=1)
     assert ei.value.status == -2
+
+
+# ---------------------------------------------------------------- maximum sizes
+def test_playouts_million_leaves_sampled(mcts, orc):
+    """1,048,576 leaves x 1 playout (one warp spans 32 leaves everywhere)."""
+    n = 1 << 20
+    d_leaves = dev.gen_positions(mcts, 5, n, 0, 50)
+    d_out = dev.empty_wdl(n)
+    mcts.playouts_async(d_leaves.data_ptr(), n, 1, 6, 0, d_out.data_ptr(), 0, None)
+    torch.cuda.synchronize()
+    wdl = d_out.cpu().numpy()
+    assert (wdl.sum(axis=1) == 1).all()
+    rng = np.random.default_rng(1)
+    idx = np.concatenate([[0, n - 1], rng.choice(n, 200, replace=False)])
+    leaves = dev.tensor_to_positions(d_leaves[torch.as_tensor(idx, device="cuda")])
+    want = orc.gen_positions(5, n, 0, 50)[idx]
+    assert (leaves == want).all()
+    for j, i in enumerate(idx):
+        owdl, _ = orc.playouts(want[j:j + 1], 1, seed=6, leaf_id_base=int(i))
+        assert wdl[i].tolist() == owdl[0].tolist(), i
+
+
+def test_search_block_4736_trees_of_32(orc):
+    """Fig. 5's largest block-32 shape: 4736 trees x 32 threads (32 CTAs per SM)."""
+    m = pkg.Mcts(c_uct=1.0, scheme="block", device=0)
+    root = orc.gen_positions(31, 1, 30, 40)
+    res = m.search(root, iterations=2, n_trees=4736, threads_per_tree=32, seed=8)
+    ostats, obest, _ = orc.uct_search(root, 4736, 32, 2, 8)
+    _cmp_search(res, ostats, obest)
+    m.close()
+
+
+def test_search_leaf_max_batch(mcts_leaf, orc):
+    """Leaf parallelism at the largest batch the API allows (65536 per leaf)."""
+    root = orc.gen_positions(32, 1, 40, 48)
+    res = mcts_leaf.search(root, iterations=2, n_trees=1, threads_per_tree=65536, seed=9)
+    ostats, obest, _ = orc.uct_search(root, 1, 65536, 2, 9)
+    _cmp_search(res, ostats, obest)
