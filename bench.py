@@ -252,7 +252,10 @@ def selfplay_leg(args, world, rank, local):
     torch.cuda.set_device(local)
     if world > 1:
         init_dist(dist, torch, local)
-    scheme = args.sp_scheme
+    hybrid = args.sp_scheme == "hybrid"
+    if hybrid and world > 1:
+        raise SystemExit("--sp-scheme hybrid is single-GPU")
+    scheme = "leaf" if args.sp_scheme == "leaf" else "block"
     n_trees, threads = (SEARCH_TREES, SEARCH_THREADS) if scheme == "block" else (1, LEAF_THREADS)
     m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
     stream = torch.cuda.current_stream()
@@ -261,6 +264,10 @@ def selfplay_leg(args, world, rank, local):
 
     def search(black, white, to_move, seed):
         pos = pkg.position(black, white, to_move)
+        if hybrid:  # NEXT-1: GPU trees + one host tree per host core, root sums merged
+            r = m.search_hybrid(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads,
+                                seed=seed, cpu_threads=len(os.sched_getaffinity(0)))
+            return r["best_move"], r["root_visits"]
         m.search_async(pos, 0, args.move_ms, n_trees, threads, seed, rank * n_trees,
                        stats.data_ptr(), stream)
         with torch.cuda.stream(stream):
@@ -290,7 +297,7 @@ def selfplay_leg(args, world, rank, local):
 
     cores = len(os.sched_getaffinity(0))
     workload = (f"configs[{2 if scheme == 'block' else 3}] searcher ({n_trees} trees x {threads} "
-                f"threads per GPU, {scheme}, {world} GPU(s))")
+                f"threads per GPU, {args.sp_scheme}, {world} GPU(s))")
     if args.fig7:
         curves = []
         t = 1
@@ -345,7 +352,7 @@ def main():
     ap.add_argument("--selfplay", type=int, default=0,
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
-    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf"])
+    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid"])
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")

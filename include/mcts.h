@@ -161,6 +161,21 @@ mcts_status mcts_search_async(mcts_handle* h, const mcts_position* root, mcts_bu
                               uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
                               uint32_t tree_id_base, int64_t* d_stats, void* stream);
 
+/* Hybrid CPU/GPU search (§III-A):
+ * the block-parallel GPU search of mcts_search_async runs while cpu_threads
+ * host threads grow one tree each from the same root with one simulation per
+ * iteration (the paper's CPU MCTS, L185-L186; Philox streams c0 = 0x40000000 +
+ * thread, c1 = iteration, c2 = 0); the root statistics of all GPU and host
+ * trees are summed (L199-L202) into out, the host trees' share alone into
+ * out_cpu (nullable). Iteration mode: every GPU tree and every host tree runs
+ * budget.iterations iterations (deterministic; host trees = the oracle's UCT
+ * with unit 1). Time mode: both sides stop at time_ms. MCTS_BLOCK handles
+ * only; errors as mcts_search plus INVALID_ARGUMENT for cpu_threads outside
+ * [1, 1024]. Synchronous. */
+mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                               uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                               uint32_t cpu_threads, mcts_root_stats* out, mcts_root_stats* out_cpu);
+
 /* Best move from a (merged) stats vector on the host: argmax of visits[0..64],
  * lowest index on ties, -1 if all zero (R8). */
 int32_t mcts_best_move(const int64_t* stats);

@@ -14,13 +14,14 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17",
-    "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
+    "-Xcompiler", "-fPIC", "-Xcompiler", "-O2", "-Xcompiler", "-ffp-contract=off", "-Xcompiler", "-pthread",
     "-shared",
 ]
 
 
 def sources() -> list:
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+                  + glob.glob(os.path.join(CSRC, "*.cpp")) + glob.glob(os.path.join(CSRC, "*.h"))
                   + [os.path.join(ROOT, "include", "mcts.h")])
 
 
@@ -38,7 +39,7 @@ def build(force: bool = False, verbose: bool = False, out: str = None, defines=(
         return LIB
     tmp = target + f".tmp{os.getpid()}"
     cmd = [NVCC, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-Xptxas", "-v",
-           os.path.join(CSRC, "mcts_api.cu"), "-o", tmp]
+           os.path.join(CSRC, "mcts_api.cu"), os.path.join(CSRC, "host_mcts.cpp"), "-o", tmp]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + res.stdout + res.stderr)

@@ -22,7 +22,7 @@ MCTS_BLOCK, MCTS_LEAF = 0, 1
 # every symbol include/mcts.h declares
 EXPORTS = (
     "mcts_create", "mcts_destroy", "mcts_playouts", "mcts_playouts_async", "mcts_search",
-    "mcts_search_async", "mcts_best_move", "mcts_gen_positions_async", "mcts_ln_table",
+    "mcts_search_async", "mcts_search_hybrid", "mcts_best_move", "mcts_gen_positions_async", "mcts_ln_table",
     "mcts_status_string", "mcts_last_error", "mcts_version",
 )
 
@@ -82,6 +82,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
     L.mcts_search.restype = i32
     L.mcts_search_async.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, vp, vp]
     L.mcts_search_async.restype = i32
+    L.mcts_search_hybrid.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, P(RootStats), P(RootStats)]
+    L.mcts_search_hybrid.restype = i32
     L.mcts_best_move.argtypes = [vp]
     L.mcts_best_move.restype = i32
     L.mcts_gen_positions_async.argtypes = [vp, u64, u32, u32, u32, vp, vp]
@@ -187,6 +189,28 @@ class Mcts:
         stats[195], stats[196], stats[197] = out.root_visits, out.iterations_done, out.plies
         return dict(stats=stats, best_move=int(out.best_move), root_visits=int(out.root_visits),
                     iterations=int(out.iterations_done), plies=int(out.plies))
+
+    @staticmethod
+    def _stats_dict(out: "RootStats") -> dict:
+        stats = np.zeros(STATS_LEN, dtype=np.int64)
+        stats[0:65] = np.ctypeslib.as_array(out.visits)
+        stats[65:130] = np.ctypeslib.as_array(out.wins)
+        stats[130:195] = np.ctypeslib.as_array(out.draws)
+        stats[195], stats[196], stats[197] = out.root_visits, out.iterations_done, out.plies
+        return dict(stats=stats, best_move=int(out.best_move), root_visits=int(out.root_visits),
+                    iterations=int(out.iterations_done), plies=int(out.plies))
+
+    def search_hybrid(self, root=None, iterations: int = 0, time_ms: float = 0.0, n_trees: int = 1,
+                      threads_per_tree: int = 64, seed: int = 1, cpu_threads: int = 1) -> dict:
+        """mcts_search_hybrid: GPU block-parallel trees + host trees, root sums merged."""
+        out, cpu = RootStats(), RootStats()
+        rp = ctypes.byref(_pos(root)) if root is not None else None
+        self._check(self.L.mcts_search_hybrid(self.h, rp, Budget(iterations, time_ms), n_trees,
+                                              threads_per_tree, seed, cpu_threads, ctypes.byref(out),
+                                              ctypes.byref(cpu)))
+        d = self._stats_dict(out)
+        d["cpu"] = self._stats_dict(cpu)
+        return d
 
     def search_async(self, root, iterations: int, time_ms: float, n_trees: int,
                      threads_per_tree: int, seed: int, tree_id_base: int, d_stats_ptr: int,

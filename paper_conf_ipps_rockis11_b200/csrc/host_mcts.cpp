@@ -1,0 +1,219 @@
+// host_mcts.cpp — host-thread UCT trees for the hybrid CPU/GPU search (see
+// host_mcts.h). Same rules, RNG streams and UCT arithmetic as the device path
+// (R1-R10) with one simulation per iteration; used only by
+// mcts_search_hybrid, never as a substitute for the GPU.
+#include "host_mcts.h"
+
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <thread>
+
+namespace mcts_host {
+namespace {
+
+typedef uint64_t u64;
+typedef uint32_t u32;
+
+constexpr u64 kInner = 0x7E7E7E7E7E7E7E7EULL;
+
+template <int S>
+inline u64 sh(u64 x) {
+  if constexpr (S > 0) return x << S;
+  else return x >> (-S);
+}
+
+template <int S>
+inline u64 dir_moves(u64 P, u64 M) {
+  u64 t = M & sh<S>(P);
+  for (int i = 0; i < 5; ++i) t |= M & sh<S>(t);
+  return sh<S>(t);
+}
+
+inline u64 legal(u64 P, u64 O) {
+  const u64 M = O & kInner;
+  u64 m = dir_moves<1>(P, M) | dir_moves<-1>(P, M) | dir_moves<8>(P, O) | dir_moves<-8>(P, O);
+  m |= dir_moves<7>(P, M) | dir_moves<-7>(P, M) | dir_moves<9>(P, M) | dir_moves<-9>(P, M);
+  return m & ~(P | O);
+}
+
+template <int S>
+inline u64 dir_flips(u64 x, u64 P, u64 M) {
+  u64 t = M & sh<S>(x);
+  for (int i = 0; i < 5; ++i) t |= M & sh<S>(t);
+  return (sh<S>(t) & P) ? t : 0ULL;
+}
+
+inline u64 flips(int sq, u64 P, u64 O) {
+  const u64 x = 1ULL << sq, M = O & kInner;
+  return dir_flips<1>(x, P, M) | dir_flips<-1>(x, P, M) | dir_flips<8>(x, P, O) |
+         dir_flips<-8>(x, P, O) | dir_flips<7>(x, P, M) | dir_flips<-7>(x, P, M) |
+         dir_flips<9>(x, P, M) | dir_flips<-9>(x, P, M);
+}
+
+inline int popc(u64 x) { return __builtin_popcountll(x); }
+
+inline int kth_bit(u64 m, u32 k) {
+  for (u32 i = 0; i < k; ++i) m &= m - 1;
+  return __builtin_ctzll(m);
+}
+
+inline void philox(u32 c[4], u32 k0, u32 k1) {
+  for (int i = 0; i < 10; ++i) {
+    const u64 p0 = (u64)0xD2511F53u * c[0], p1 = (u64)0xCD9E8D57u * c[2];
+    const u32 n0 = (u32)(p1 >> 32) ^ c[1] ^ k0, n2 = (u32)(p0 >> 32) ^ c[3] ^ k1;
+    c[1] = (u32)p1;
+    c[3] = (u32)p0;
+    c[0] = n0;
+    c[2] = n2;
+    k0 += 0x9E3779B9u;
+    k1 += 0xBB67AE85u;
+  }
+}
+
+// One random playout; +1 / 0 / -1 for the side to move at the start.
+int playout(u64 me, u64 op, u64 seed, u32 c0, u32 c1, u32 c2, u64* plies) {
+  u32 buf[4] = {0, 0, 0, 0};
+  u32 w = 0;
+  bool start = true, passed = false;
+  for (;;) {
+    const u64 m = legal(me, op);
+    if (m == 0) {
+      if (passed) break;
+      passed = true;
+    } else {
+      passed = false;
+      if ((w & 3u) == 0u) {
+        buf[0] = c0; buf[1] = c1; buf[2] = c2; buf[3] = w >> 2;
+        philox(buf, (u32)seed, (u32)(seed >> 32));
+      }
+      const u32 r = buf[w & 3u];
+      ++w;
+      const int sq = kth_bit(m, (u32)(((u64)r * (u32)popc(m)) >> 32));
+      const u64 f = flips(sq, me, op);
+      me |= f | (1ULL << sq);
+      op &= ~f;
+      ++*plies;
+    }
+    const u64 t = me; me = op; op = t;
+    start = !start;
+  }
+  const int a = popc(start ? me : op), b = popc(start ? op : me);
+  return (a > b) - (a < b);
+}
+
+struct Tree {
+  std::vector<u64> own, opp, lg;
+  std::vector<u32> k, w, d, first, nchild, limit, move;
+  std::vector<uint8_t> term;
+  void add(u64 o, u64 p, u32 mv) {
+    const u64 l = legal(o, p);
+    const bool t = l == 0 && legal(p, o) == 0;
+    own.push_back(o); opp.push_back(p); lg.push_back(l);
+    k.push_back(0); w.push_back(0); d.push_back(0);
+    first.push_back(0xFFFFFFFFu); nchild.push_back(0);
+    limit.push_back(t ? 0u : (l ? (u32)popc(l) : 1u));
+    move.push_back(mv); term.push_back(t ? 1 : 0);
+  }
+};
+
+void run_tree(const HostSearchArgs& a, u32 t, int64_t* st) {
+  Tree T;
+  T.add(a.own, a.opp, 0xFFu);
+  if (T.term[0]) return;
+  u64 plies = 0;
+  u64 it = 0;
+  std::vector<u32> path;
+  for (; it < a.iterations; ++it) {
+    if (a.deadline_ns && (it & 15u) == 0 &&
+        std::chrono::steady_clock::now().time_since_epoch().count() >= a.deadline_ns)
+      break;
+    path.clear();
+    u32 v = 0;
+    path.push_back(v);
+    while (!T.term[v] && T.nchild[v] >= T.limit[v]) {  // selection
+      const double lnp = a.lnT[T.k[v]];
+      u32 best = 0;
+      double bu = -INFINITY;
+      for (u32 i = 0; i < T.nchild[v]; ++i) {
+        const u32 c = T.first[v] + i;
+        const double n = (double)T.k[c];  // unit = 1: n = k
+        const double u = (double)T.w[c] / n + a.C * std::sqrt(lnp / n);
+        if (u > bu) { bu = u; best = c; }
+      }
+      v = best;
+      path.push_back(v);
+    }
+    if (!T.term[v]) {  // expansion: children stored in a reserved contiguous block
+      if (T.nchild[v] == 0) {
+        T.first[v] = (u32)T.own.size();
+        for (u32 i = 0; i < T.limit[v]; ++i) T.add(0, 0, 0);  // placeholders
+      }
+      const u32 c = T.first[v] + T.nchild[v];
+      const u64 o = T.own[v], p = T.opp[v], l = T.lg[v];
+      u64 co, cp;
+      u32 mv;
+      if (l == 0) { co = p; cp = o; mv = 64; }
+      else {
+        const int sq = kth_bit(l, T.nchild[v]);
+        const u64 f = flips(sq, o, p);
+        co = p & ~f; cp = o | f | (1ULL << sq); mv = (u32)sq;
+      }
+      const u64 cl = legal(co, cp);
+      const bool ct = cl == 0 && legal(cp, co) == 0;
+      T.own[c] = co; T.opp[c] = cp; T.lg[c] = cl; T.move[c] = mv; T.term[c] = ct ? 1 : 0;
+      T.limit[c] = ct ? 0u : (cl ? (u32)popc(cl) : 1u);
+      T.nchild[v] += 1;
+      v = c;
+      path.push_back(v);
+    }
+    int r;  // simulation (one per iteration)
+    if (T.term[v]) {
+      const int x = popc(T.own[v]), y = popc(T.opp[v]);
+      r = (x > y) - (x < y);
+    } else {
+      r = playout(T.own[v], T.opp[v], a.seed, a.tree_id_base + t, (u32)it, 0u, &plies);
+    }
+    u32 mover_wins = r < 0, other_wins = r > 0;  // backpropagation
+    const u32 draw = r == 0;
+    for (size_t i = path.size(); i-- > 0;) {
+      const u32 x = path[i];
+      T.k[x] += 1; T.w[x] += mover_wins; T.d[x] += draw;
+      std::swap(mover_wins, other_wins);
+    }
+  }
+  // root children -> stats (int64 sums, layout of include/mcts.h MCTS_STATS_LEN)
+  for (u32 i = 0; i < T.nchild[0]; ++i) {
+    const u32 c = T.first[0] + i;
+    st[T.move[c]] += T.k[c];
+    st[65 + T.move[c]] += T.w[c];
+    st[130 + T.move[c]] += T.d[c];
+  }
+  st[195] += T.k[0];
+  st[196] += (int64_t)it;
+  st[197] += (int64_t)plies;
+}
+
+}  // namespace
+
+void search(const HostSearchArgs& a, int64_t* stats) {
+  for (int i = 0; i < 198; ++i) stats[i] = 0;
+  const u32 T = a.threads ? a.threads : 1;
+  std::vector<std::vector<int64_t>> part(T, std::vector<int64_t>(198, 0));
+  std::atomic<u32> next{0};
+  auto worker = [&](u32 tid) {
+    for (;;) {
+      const u32 t = next.fetch_add(1);
+      if (t >= a.n_trees) break;
+      run_tree(a, t, part[tid].data());
+    }
+  };
+  std::vector<std::thread> pool;
+  for (u32 i = 1; i < T; ++i) pool.emplace_back(worker, i);
+  worker(0);
+  for (auto& th : pool) th.join();
+  for (u32 i = 0; i < T; ++i)
+    for (int j = 0; j < 198; ++j) stats[j] += part[i][j];
+}
+
+}  // namespace mcts_host

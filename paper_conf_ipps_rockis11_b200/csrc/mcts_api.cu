@@ -3,16 +3,21 @@
 // Host side only marshals arguments, validates them, owns device scratch
 // (tree pools, ln tables, staging) and launches kernels; every step of the hot
 // path runs on the GPU. There is no CPU fallback: without an sm_100 device the
-// compute calls fail with MCTS_E_NO_DEVICE.
+// compute calls fail with MCTS_E_NO_DEVICE. The one place host threads compute
+// is mcts_search_hybrid, the paper's hybrid scheme, where they grow additional
+// trees *alongside* a running GPU search (host_mcts.cpp).
 #include <cuda_runtime.h>
 
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "../../include/mcts.h"
 #include "kernels.cuh"
+#include "host_mcts.h"
 
 using namespace mcts_dev;
 
@@ -54,6 +59,7 @@ struct mcts_handle {
   u64* d_rays = nullptr;      // ray table for the flip kernels (kRayTable u64)
   u32* d_work = nullptr;      // playout work counter
   int playout_ctas = 0;       // resident playout CTAs (SMs x occupancy)
+  std::vector<double> host_lnT1;  // RN(ln k) for the hybrid's host trees
 };
 
 namespace {
@@ -434,6 +440,76 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   out->plies = (uint64_t)hs[197];
   out->best_move = mcts_best_move((const int64_t*)hs);
   out->reserved = 0;
+  return MCTS_OK;
+}
+
+static void fill_root_stats(const long long* hs, mcts_root_stats* out) {
+  for (int i = 0; i < 65; ++i) {
+    out->visits[i] = (uint64_t)hs[i];
+    out->wins[i] = (uint64_t)hs[65 + i];
+    out->draws[i] = (uint64_t)hs[130 + i];
+  }
+  out->root_visits = (uint64_t)hs[195];
+  out->iterations_done = (uint64_t)hs[196];
+  out->plies = (uint64_t)hs[197];
+  out->best_move = mcts_best_move((const int64_t*)hs);
+  out->reserved = 0;
+}
+
+mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                               uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                               uint32_t cpu_threads, mcts_root_stats* out, mcts_root_stats* out_cpu) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (!out) return fail(h, MCTS_E_INVALID_ARGUMENT, "out == NULL");
+  if (h->params.scheme != MCTS_BLOCK) return fail(h, MCTS_E_INVALID_ARGUMENT, "hybrid search needs MCTS_BLOCK");
+  if (cpu_threads == 0 || cpu_threads > 1024) return fail(h, MCTS_E_INVALID_ARGUMENT, "cpu_threads must be in [1, 1024]");
+  const mcts_position* rp = root ? root : (h->has_position ? &h->position : nullptr);
+  if (!rp) return fail(h, MCTS_E_INVALID_ARGUMENT, "no root position");
+  if (!position_ok(*rp)) return fail(h, MCTS_E_INVALID_POSITION, "root: black & white overlap or bad to_move");
+  const bool by_time = budget.time_ms != 0.0;
+  const uint64_t host_k = by_time ? (1u << 20) : budget.iterations;
+  if (!by_time && (host_k == 0 || host_k > (1u << 24)))
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "iterations must be in [1, 2^24]");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  // Host ln table lnT[k] = RN(ln k) (unit = 1), generated by the device kernel.
+  if (h->host_lnT1.size() < host_k + 1) {
+    double* d = nullptr;
+    const size_t n = (size_t)host_k + 1;
+    CK(h, cudaMalloc(&d, n * sizeof(double)));
+    ln_table_kernel<<<(unsigned)((n + 255) / 256), 256, 0, h->stream>>>(d, 1u, (u32)host_k);
+    std::vector<double> tmp(n);
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaMemcpyAsync(tmp.data(), d, n * sizeof(double), cudaMemcpyDeviceToHost, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+    cudaFree(d);
+    if (e != cudaSuccess) return cuda_fail(h, e, "host ln table");
+    h->host_lnT1.swap(tmp);
+  }
+  // GPU trees (async), then the host trees in this thread's pool while the
+  // kernel runs; host tree ids start at 0x40000000 so no stream is shared.
+  st = search_impl(h, rp, budget, n_trees, threads_per_tree, seed, 0, h->d_stats, h->stream);
+  if (st) return st;
+  const int64_t start_ns = std::chrono::steady_clock::now().time_since_epoch().count();
+  mcts_host::HostSearchArgs a;
+  a.own = rp->to_move ? rp->white : rp->black;
+  a.opp = rp->to_move ? rp->black : rp->white;
+  a.seed = seed;
+  a.C = h->params.c_uct;
+  a.n_trees = cpu_threads;
+  a.tree_id_base = 0x40000000u;
+  a.iterations = host_k;
+  a.deadline_ns = by_time ? start_ns + (int64_t)llround(budget.time_ms * 1e6) : 0;
+  a.threads = cpu_threads;
+  a.lnT = h->host_lnT1.data();
+  long long cs[MCTS_STATS_LEN];
+  mcts_host::search(a, (int64_t*)cs);
+  long long hs[MCTS_STATS_LEN];
+  CK(h, cudaMemcpyAsync(hs, h->d_stats, sizeof(hs), cudaMemcpyDeviceToHost, h->stream));
+  CK(h, cudaStreamSynchronize(h->stream));
+  if (out_cpu) fill_root_stats(cs, out_cpu);
+  for (int i = 0; i < MCTS_STATS_LEN; ++i) hs[i] += cs[i];  // root sum over all trees (L199-L202)
+  fill_root_stats(hs, out);
   return MCTS_OK;
 }
 

@@ -298,3 +298,30 @@ def test_search_leaf_max_batch(mcts_leaf, orc):
     res = mcts_leaf.search(root, iterations=2, n_trees=1, threads_per_tree=65536, seed=9)
     ostats, obest, _ = orc.uct_search(root, 1, 65536, 2, 9)
     _cmp_search(res, ostats, obest)
+
+
+# ---------------------------------------------------------------- hybrid (NEXT-1)
+def test_search_hybrid_iteration_mode(mcts, orc):
+    """GPU trees + host trees (c0 = 0x40000000 + t, unit 1), root sums merged:
+    equal to the oracle's two searches added up, bit for bit."""
+    root = orc.gen_positions(41, 1, 20, 30)
+    res = mcts.search_hybrid(root, iterations=40, n_trees=6, threads_per_tree=64, seed=12, cpu_threads=3)
+    g, _, gp = orc.uct_search(root, 6, 64, 40, 12)
+    c, _, cp = orc.uct_search(root, 3, 1, 40, 12, tree_id_base=0x40000000)
+    assert res["cpu"]["stats"][:197].tolist() == c[:197].tolist()
+    assert res["cpu"]["plies"] == cp
+    merged = g + c
+    assert res["stats"][:197].tolist() == merged[:197].tolist()
+    assert res["best_move"] == int(np.argmax(merged[:65]))
+    assert res["plies"] == gp + cp
+
+
+def test_search_hybrid_time_mode(mcts, orc):
+    root = orc.gen_positions(42, 1, 10, 20)
+    res = mcts.search_hybrid(root, time_ms=50.0, n_trees=148, threads_per_tree=128, seed=3, cpu_threads=4)
+    cpu = res["cpu"]["stats"]
+    assert cpu[196] > 4 and cpu[195] == cpu[196]  # unit 1: one playout per iteration
+    s = res["stats"]
+    assert s[:65].sum() == s[195]
+    own, opp = pkg.own_opp(root)
+    assert (orc.legal(own, opp) >> res["best_move"]) & 1
