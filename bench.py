@@ -71,6 +71,21 @@ def clocks_summary(path, gpu_index):
             "samples": len(rows)}
 
 
+def integer_peak():
+    """Integer roofline denominator: the measured B200 rate of an
+    alternating LOP3/IMAD stream (both integer pipes, i.e. the issue limit) from
+    tools/int_peaks.cu (profiles/int_peaks.json), else the issue-slot count
+    148 SM x 4 SMSP x 32 lanes x sm_max_mhz. Also returns the ALU-pipe-only rate."""
+    try:
+        ip = json.load(open(os.path.join(ROOT, "profiles", "int_peaks.json")))
+        return (ip["lop3_imad_mixed"], "measured: alternating LOP3/IMAD stream, all SMs "
+                "(tools/int_peaks.cu -> profiles/int_peaks.json)", ip["lop3_alu"])
+    except Exception:
+        sm_max = measured_peaks().get("sm_max_mhz", 1965.0)
+        return (148 * 4 * 32 * sm_max * 1e6, f"derived: 148 SM x 4 SMSP x 32 lanes x {sm_max:.0f} MHz",
+                148 * 4 * 16 * sm_max * 1e6)
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -503,7 +518,7 @@ def main():
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
             # same per-ply op model as the headline roofline, per GPU
             "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ALG_OPS_PER_PLY
-                             / (148 * 4 * 32 * measured_peaks().get("sm_max_mhz", 1965.0) * 1e6),
+                             / integer_peak()[0],
         }
         log('ml = pkg.Mcts(')
         ml = pkg.Mcts(c_uct=1.0, scheme="leaf", device=local)
@@ -528,9 +543,7 @@ def main():
             dist.destroy_process_group()
         return
 
-    peaks = measured_peaks()
-    sm_max = peaks.get("sm_max_mhz", 1965.0)
-    peak_ops = 148 * 4 * 32 * sm_max * 1e6  # thread-instruction issue slots / s
+    peak_ops, peak_basis, alu_peak = integer_peak()
     kern_s = kernel_ms / 1e3 / args.steps
     plies_per_launch = plies_local / args.steps
     achieved = plies_per_launch * ALG_OPS_PER_PLY / kern_s
@@ -557,8 +570,7 @@ def main():
         "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak_ops / 1e9,
                      "unit": "Gop/s", "frac": achieved / peak_ops, "traffic": traffic,
                      "ops_per_ply": ALG_OPS_PER_PLY, "plies_per_launch": plies_per_launch, "ncu": ncu,
-                     "peak_basis": f"issue slots 148 SM x 4 SMSP x 32 lanes x {sm_max:.0f} MHz "
-                                   "(MEASURED_PEAKS.json sm_max_mhz), DESIGN.md §6"},
+                     "peak_basis": peak_basis, "alu_pipe_peak": alu_peak / 1e9},
         "e2e": {"value": e2e_value, "unit": "playouts/s",
                 "h2d_bytes_per_step": N_LEAVES * 24, "d2h_bytes_per_step": N_LEAVES * 12 + 8,
                 "api": "mcts_playouts (host buffers, pinned)"},
