@@ -21,7 +21,10 @@
  *   - Ownership: the caller owns every input/output buffer (host or device as
  *     each argument states). The handle owns its device scratch (tree pools,
  *     ln table, staging) and frees it in mcts_destroy.
- *   - A handle is not thread-safe; use one per host thread / rank.
+ *   - A handle is not thread-safe; use one per host thread / rank. Playout
+ *     launches on one handle may overlap on different streams (each launch
+ *     takes its own scratch, up to 256 in flight); searches may not overlap
+ *     another search of the same handle (they share its tree pool).
  *   - Errors: no exception crosses the ABI; every function returns an
  *     mcts_status (< 0 on error) and mcts_last_error() gives the text.
  *   - Streams are passed as `void*` holding a cudaStream_t (NULL = the legacy

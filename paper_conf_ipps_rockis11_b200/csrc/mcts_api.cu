@@ -24,6 +24,10 @@ using namespace mcts_dev;
 static_assert(sizeof(mcts_position) == sizeof(DevPosition), "position layout");
 static_assert(sizeof(mcts_wdl) == sizeof(WdlOut), "wdl layout");
 
+// Playout launches take a fresh work counter from a ring, so concurrent launches
+// on different streams of one handle (up to kWorkSlots in flight) never share one.
+constexpr uint32_t kWorkSlots = 256;
+
 struct mcts_handle {
   int device = 0;
   mcts_params params{};
@@ -57,7 +61,8 @@ struct mcts_handle {
   int* d_error = nullptr;
   LeafSync* d_leafsync = nullptr;
   u64* d_rays = nullptr;      // ray table for the flip kernels (kRayTable u64)
-  u32* d_work = nullptr;      // playout work counter
+  u32* d_work = nullptr;      // ring of playout work counters (one per launch)
+  uint32_t work_slot = 0;
   int playout_ctas = 0;       // resident playout CTAs (SMs x occupancy)
   std::vector<double> host_lnT1;  // RN(ln k) for the hybrid's host trees
 };
@@ -304,7 +309,7 @@ mcts_status mcts_create(const mcts_position* position, const mcts_params* params
   if (e == cudaSuccess) e = cudaMalloc(&h->d_plies, sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_leafsync, sizeof(LeafSync));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_rays, kRayTable * sizeof(u64));
-  if (e == cudaSuccess) e = cudaMalloc(&h->d_work, sizeof(u32));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_work, kWorkSlots * sizeof(u32));
   if (e == cudaSuccess) {
     rays_init_kernel<<<1, 256, 0, h->stream>>>(h->d_rays);
     e = cudaGetLastError();
@@ -359,10 +364,12 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
   if ((total + 31) / 32 > 0xFFFFFFF0ull) return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large (>= 2^37 playouts)");
   const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
   const unsigned blocks = (unsigned)(need < (uint64_t)h->playout_ctas ? need : (uint64_t)h->playout_ctas);
-  CK(h, cudaMemsetAsync(h->d_work, 0, sizeof(u32), s));
+  // a fresh counter per launch, so launches on different streams do not share one
+  u32* work = h->d_work + (h->work_slot++ % kWorkSlots);
+  CK(h, cudaMemsetAsync(work, 0, sizeof(u32), s));
   playouts_kernel<<<blocks, kPlayoutThreads, 0, s>>>(
       (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), leaf_id_base, (WdlOut*)d_out,
-      (unsigned long long*)d_plies, h->d_rays, h->d_work);
+      (unsigned long long*)d_plies, h->d_rays, work);
   CK(h, cudaGetLastError());
   return MCTS_OK;
 }

@@ -325,3 +325,20 @@ def test_search_hybrid_time_mode(mcts, orc):
     assert s[:65].sum() == s[195]
     own, opp = pkg.own_opp(root)
     assert (orc.legal(own, opp) >> res["best_move"]) & 1
+
+
+def test_playouts_concurrent_streams(mcts, orc):
+    """Two launches of one handle on two streams overlap safely (per-launch scratch)."""
+    n, per = 300, 64
+    d_a = dev.gen_positions(mcts, 51, n, 20, 40)
+    d_b = dev.gen_positions(mcts, 52, n, 20, 40)
+    torch.cuda.synchronize()
+    out_a, out_b = dev.empty_wdl(n), dev.empty_wdl(n)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    for _ in range(3):
+        mcts.playouts_async(d_a.data_ptr(), n, per, 5, 0, out_a.data_ptr(), 0, s1)
+        mcts.playouts_async(d_b.data_ptr(), n, per, 6, 0, out_b.data_ptr(), 0, s2)
+    torch.cuda.synchronize()
+    wa, _ = orc.playouts(orc.gen_positions(51, n, 20, 40), per, seed=5)
+    wb, _ = orc.playouts(orc.gen_positions(52, n, 20, 40), per, seed=6)
+    assert (out_a.cpu().numpy() == wa).all() and (out_b.cpu().numpy() == wb).all()

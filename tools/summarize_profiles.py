@@ -61,6 +61,9 @@ if os.path.exists(launch_csv):
     with open(os.path.join(out_dir, f"{tag}_launches.txt"), "w") as f:
         f.write("# ncu --metrics gpu__time_duration.sum --clock-control none, bench.py --steps 5 --warmup 3\n")
         f.write("# (cold-cache serialised launches: compare shares, not absolutes)\n")
+        f.write("# at::...FillFunctor<unsigned char> = the 256 MiB L2 flush between timed steps (outside\n"
+                "# the timed events); ln_table / gen_positions / rays_init = one-time setup; search kernels\n"
+                "# here run in time mode under ncu serialisation (their deadline passes) and are not the step\n")
         allt = sum(t for _, t in tot.values())
         for name, (n, t) in sorted(tot.items(), key=lambda kv: -kv[1][1]):
             f.write(f"{name:60s} launches {n:5d}  total {t/1e3:12.1f} us  share {100*t/allt:5.1f}%\n")
