@@ -22,7 +22,6 @@ import os
 import subprocess
 import sys
 import tempfile
-import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -394,7 +393,6 @@ def main():
     if args.warmup < 3:
         args.warmup = 3
 
-    import numpy as np
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_rockis11_b200 as pkg
@@ -465,7 +463,6 @@ def main():
 
     log('# ---- end to end')
     # ---- end to end through the C ABI with host buffers (H2D + kernel + D2H)
-    from paper_conf_ipps_rockis11_b200.positions import own_opp  # noqa: F401
     h_leaves = torch.empty((N_LEAVES, 3), dtype=torch.int64).pin_memory()
     h_leaves.copy_(d_leaves.cpu())
     h_out = torch.empty((N_LEAVES, 3), dtype=torch.int32).pin_memory()

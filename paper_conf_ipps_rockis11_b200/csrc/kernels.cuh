@@ -122,7 +122,6 @@ struct SearchArgs {
   const u64* rays;       // global ray table (kRayTable u64)
 };
 
-constexpr int kSearchThreadsMax = 1024;
 
 template <int MAX_THREADS, int MIN_BLOCKS>
 __global__ void __launch_bounds__(MAX_THREADS, MIN_BLOCKS)

@@ -42,8 +42,6 @@ struct mcts_handle {
   WdlOut* d_wdl = nullptr;
   size_t wdl_cap = 0;
   unsigned long long* d_plies = nullptr;
-  void* h_pinned = nullptr;
-  size_t pinned_cap = 0;
 
   // trees
   void* pool_mem = nullptr;
@@ -344,7 +342,6 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_leafsync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
-  if (h->h_pinned) cudaFreeHost(h->h_pinned);
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
