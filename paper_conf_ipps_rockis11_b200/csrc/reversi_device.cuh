@@ -27,6 +27,9 @@
 #ifndef MCTS_EAST_F
 #define MCTS_EAST_F 1    // horizontal carry moves with IMAD shifts/adds
 #endif
+#ifndef MCTS_FLIP_WIDE
+#define MCTS_FLIP_WIDE 0 // flip carries with IMAD.WIDE instead of IADD3 pairs
+#endif
 
 namespace mcts_dev {
 
@@ -285,7 +288,17 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
 // non-ray bits, all ones) and lands on the first non-opponent ray square.
 // run = ray squares that carried (~s & O & m); kept iff the landing square is P.
 __device__ __forceinline__ void up_flips(u64& f, u64 first, u64 P, u64 O, u64 m) {
-  const u64 s = (O | ~m) + first;
+  const u64 xo = O | ~m;
+#if MCTS_FLIP_WIDE
+  // xo + first on the FMA pipe: IMAD for the high words, then one IMAD.WIDE
+  // (xo_lo * 1 + {first_lo, xo_hi + first_hi}) carries the low word into them.
+  const u32 one = c_pow2[0];
+  const u32 hi = (u32)(first >> 32) * one + (u32)(xo >> 32);
+  u64 s;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(s) : "r"((u32)xo), "r"(one), "l"(join32((u32)first, hi)));
+#else
+  const u64 s = xo + first;
+#endif
   if (s & m & P) f |= ~s & O & m;
 }
 

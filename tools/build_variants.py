@@ -11,6 +11,7 @@ VARIANTS = {
     "no_upd_f": ["MCTS_UPD_F=0"],
     "no_east_f": ["MCTS_EAST_F=0"],
     "t128": ["MCTS_PLAYOUT_THREADS=128"],
+    "flip_wide": ["MCTS_FLIP_WIDE=1"],
 }
 
 if __name__ == "__main__":
