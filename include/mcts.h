@@ -192,6 +192,15 @@ int32_t mcts_best_move(const int64_t* stats);
 mcts_status mcts_gen_positions_async(mcts_handle* h, uint64_t seed, uint32_t n, uint32_t lmin,
                                      uint32_t lmax, mcts_position* d_out, void* stream);
 
+/* Perft: number of leaves of the move tree of `position` at `depth` plies
+ * (a game-over node before that counts 1; a pass counts as a ply iff
+ * pass_is_ply), computed on the device with the playout kernels' move
+ * generator and flips — pins them to the known counts (north_star: 4, 12, 56,
+ * 244, 1396, 8200, 55092, 390216 from the opening). depth <= 16; *out (host).
+ * Errors: INVALID_ARGUMENT, INVALID_POSITION, OOM (frontier > 2^20), CUDA. */
+mcts_status mcts_perft(mcts_handle* h, const mcts_position* position, uint32_t depth,
+                       uint32_t pass_is_ply, uint64_t* out);
+
 /* The device ln table used by UCT selection (R9): out[k] = RN(ln(k * unit))
  * for k = 1..K, out[0] = 0. out is a host array of K + 1 doubles. */
 mcts_status mcts_ln_table(mcts_handle* h, uint32_t unit, uint32_t K, double* out);

@@ -22,7 +22,7 @@ MCTS_BLOCK, MCTS_LEAF = 0, 1
 # every symbol include/mcts.h declares
 EXPORTS = (
     "mcts_create", "mcts_destroy", "mcts_playouts", "mcts_playouts_async", "mcts_search",
-    "mcts_search_async", "mcts_search_hybrid", "mcts_best_move", "mcts_gen_positions_async", "mcts_ln_table",
+    "mcts_search_async", "mcts_search_hybrid", "mcts_best_move", "mcts_perft", "mcts_gen_positions_async", "mcts_ln_table",
     "mcts_status_string", "mcts_last_error", "mcts_version",
 )
 
@@ -84,6 +84,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
     L.mcts_search_async.restype = i32
     L.mcts_search_hybrid.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, P(RootStats), P(RootStats)]
     L.mcts_search_hybrid.restype = i32
+    L.mcts_perft.argtypes = [vp, P(Position), u32, u32, P(u64)]
+    L.mcts_perft.restype = i32
     L.mcts_best_move.argtypes = [vp]
     L.mcts_best_move.restype = i32
     L.mcts_gen_positions_async.argtypes = [vp, u64, u32, u32, u32, vp, vp]
@@ -225,6 +227,12 @@ class Mcts:
                             stream=None):
         self._check(self.L.mcts_gen_positions_async(self.h, seed, n, lmin, lmax, d_out_ptr,
                                                     _stream_ptr(stream)))
+
+    def perft(self, position, depth: int, pass_is_ply: bool = True) -> int:
+        out = ctypes.c_uint64(0)
+        self._check(self.L.mcts_perft(self.h, ctypes.byref(_pos(position)), depth, int(pass_is_ply),
+                                      ctypes.byref(out)))
+        return int(out.value)
 
     def ln_table(self, unit: int, K: int) -> np.ndarray:
         out = np.zeros(K + 1, dtype=np.float64)

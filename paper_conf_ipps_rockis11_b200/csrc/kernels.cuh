@@ -299,6 +299,93 @@ __global__ void ln_table_kernel(double* __restrict__ out, u32 unit, u32 K) {
 
 __global__ void stamp_kernel(u64* t0) { *t0 = globaltimer_ns(); }
 
+// ---------------------------------------------------------------------------
+// Perft (leaf count of the move tree to a given depth) with the hot-loop move
+// generator and flips (legal_moves_hot / flips_hot), to pin them directly to
+// the north_star perft counts. Stage 1 (one thread) lists the frontier at
+// depth `split`; stage 2 runs one depth-first search per frontier node with an
+// explicit stack. A game-over node before the depth counts 1; a pass consumes
+// a ply iff pass_is_ply (R11).
+// ---------------------------------------------------------------------------
+struct PerftNode {
+  u64 own, opp;
+  u32 depth;  // remaining depth
+  u32 pad;
+};
+
+__device__ __forceinline__ u64 perft_moves(u64 P, u64 O) {
+  return legal_moves_hot(P, O, __brevll(P), __brevll(O));
+}
+
+// Depth-first leaf count from (own, opp) with `depth` plies to go. Nodes whose
+// remaining depth reaches `stop_at` (stage 1) are written to `frontier`
+// instead of expanded. Stack frames hold a node and its untried moves, so the
+// stack depth is at most 2 * depth + 1 (pass frames included).
+__device__ unsigned long long perft_dfs(u64 own, u64 opp, u32 depth, u32 pass_is_ply, u32 stop_at,
+                                        const u64* rays, PerftNode* frontier, u32 cap, u32* count) {
+  struct F { u64 own, opp, moves; u32 depth, pass; };
+  F st[2 * 16 + 2];
+  int sp = 0;
+  unsigned long long cnt = 0;
+  auto push = [&](u64 o, u64 p, u32 d) {
+    if (d == 0) { ++cnt; return; }
+    if (d == stop_at) {
+      const u32 k = atomicAdd(count, 1u);
+      if (k < cap) frontier[k] = {o, p, d, 0};
+      return;
+    }
+    const u64 m = perft_moves(o, p);
+    if (m == 0ULL) {
+      if (perft_moves(p, o) == 0ULL) { ++cnt; return; }  // game over: a leaf
+      st[sp++] = {o, p, 0ULL, d, 1u};                     // pass
+      return;
+    }
+    if (d == 1) { cnt += (u32)__popcll(m); return; }
+    st[sp++] = {o, p, m, d, 0u};
+  };
+  push(own, opp, depth);
+  while (sp > 0) {
+    F& f = st[sp - 1];
+    if (f.pass) {
+      const F c = f;
+      --sp;
+      push(c.opp, c.own, pass_is_ply ? c.depth - 1 : c.depth);
+      continue;
+    }
+    if (f.moves == 0ULL) { --sp; continue; }
+    const int sq = __ffsll((long long)f.moves) - 1;
+    f.moves &= f.moves - 1;
+    const u64 fl = flips_hot(sq, f.own, f.opp, __brevll(f.own), __brevll(f.opp), rays);
+    const u64 o = f.opp & ~fl, p = f.own | fl | (1ULL << sq);
+    push(o, p, f.depth - 1);
+  }
+  return cnt;
+}
+
+__global__ void perft_frontier_kernel(u64 own, u64 opp, u32 depth, u32 stop_at, u32 pass_is_ply,
+                                      const u64* __restrict__ g_rays, PerftNode* out, u32 cap,
+                                      u32* count, unsigned long long* leaves) {
+  __shared__ u64 s_rays[kRayTable];
+  load_rays(s_rays, g_rays);
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  const unsigned long long c = perft_dfs(own, opp, depth, pass_is_ply, stop_at, s_rays, out, cap, count);
+  atomicAdd(leaves, c);
+}
+
+__global__ void perft_dfs_kernel(const PerftNode* __restrict__ nodes, u32 n, u32 pass_is_ply,
+                                 const u64* __restrict__ g_rays, unsigned long long* leaves) {
+  __shared__ u64 s_rays[kRayTable];
+  load_rays(s_rays, g_rays);
+  __syncthreads();
+  const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const PerftNode v = nodes[i];
+  const unsigned long long c = perft_dfs(v.own, v.opp, v.depth, pass_is_ply, 0xFFFFFFFFu, s_rays,
+                                         nullptr, 0, nullptr);
+  if (c) atomicAdd(leaves, c);
+}
+
 // Synthetic positions, one thread per position.
 __global__ void gen_positions_kernel(uint2 key, u32 n, u32 lmin, u32 lmax, DevPosition* out) {
   const u32 p = blockIdx.x * blockDim.x + threadIdx.x;

@@ -517,6 +517,54 @@ mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_b
   return MCTS_OK;
 }
 
+mcts_status mcts_perft(mcts_handle* h, const mcts_position* position, uint32_t depth,
+                       uint32_t pass_is_ply, uint64_t* out) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (!position || !out) return fail(h, MCTS_E_INVALID_ARGUMENT, "position / out is NULL");
+  if (!position_ok(*position)) return fail(h, MCTS_E_INVALID_POSITION, "position: black & white overlap or bad to_move");
+  if (depth > 16) return fail(h, MCTS_E_INVALID_ARGUMENT, "depth must be <= 16");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  const u64 own = position->to_move ? position->white : position->black;
+  const u64 opp = position->to_move ? position->black : position->white;
+  const u32 split = 5;  // frontier at 5 plies, one depth-first search per node
+  const u32 stop_at = depth > split ? depth - split : 0xFFFFFFFFu;
+  const u32 cap = 1u << 20;
+  PerftNode* d_nodes = nullptr;
+  u32* d_count = nullptr;
+  unsigned long long* d_leaves = nullptr;
+  cudaError_t e = cudaMalloc(&d_nodes, (size_t)cap * sizeof(PerftNode));
+  if (e == cudaSuccess) e = cudaMalloc(&d_count, sizeof(u32));
+  if (e == cudaSuccess) e = cudaMalloc(&d_leaves, sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_count, 0, sizeof(u32), h->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_leaves, 0, sizeof(unsigned long long), h->stream);
+  u32 n = 0;
+  if (e == cudaSuccess) {
+    perft_frontier_kernel<<<1, 128, 0, h->stream>>>(own, opp, depth, stop_at, pass_is_ply ? 1u : 0u,
+                                                    h->d_rays, d_nodes, cap, d_count, d_leaves);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&n, d_count, sizeof(u32), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess && n > cap) {
+    cudaFree(d_nodes); cudaFree(d_count); cudaFree(d_leaves);
+    return fail(h, MCTS_E_OOM, "perft frontier exceeds 2^20 nodes");
+  }
+  if (e == cudaSuccess && n > 0) {
+    perft_dfs_kernel<<<(n + 127) / 128, 128, 0, h->stream>>>(d_nodes, n, pass_is_ply ? 1u : 0u, h->d_rays, d_leaves);
+    e = cudaGetLastError();
+  }
+  unsigned long long leaves = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&leaves, d_leaves, sizeof(leaves), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  cudaFree(d_nodes);
+  cudaFree(d_count);
+  cudaFree(d_leaves);
+  if (e != cudaSuccess) return cuda_fail(h, e, "mcts_perft");
+  *out = leaves;
+  return MCTS_OK;
+}
+
 mcts_status mcts_gen_positions_async(mcts_handle* h, uint64_t seed, uint32_t n, uint32_t lmin,
                                      uint32_t lmax, mcts_position* d_out, void* stream) {
   if (!h) return MCTS_E_INVALID_ARGUMENT;

@@ -342,3 +342,28 @@ def test_playouts_concurrent_streams(mcts, orc):
     wa, _ = orc.playouts(orc.gen_positions(51, n, 20, 40), per, seed=5)
     wb, _ = orc.playouts(orc.gen_positions(52, n, 20, 40), per, seed=6)
     assert (out_a.cpu().numpy() == wa).all() and (out_b.cpu().numpy() == wb).all()
+
+
+# ---------------------------------------------------------------- perft (device move generator)
+def _golden_perft():
+    import os
+    rows = []
+    for line in open(os.path.join(os.path.dirname(__file__), "golden", "perft_opening.txt")):
+        if line.strip() and not line.startswith("#"):
+            rows.append(tuple(int(x) for x in line.split()))
+    return rows
+
+
+@pytest.mark.parametrize("depth,with_pass,without_pass", _golden_perft())
+def test_device_perft_opening(mcts, depth, with_pass, without_pass):
+    """The hot-loop move generator and flips against the north_star perft counts."""
+    assert mcts.perft(pkg.opening(), depth, True) == with_pass
+    assert mcts.perft(pkg.opening(), depth, False) == without_pass
+
+
+def test_device_perft_random_positions(mcts, orc):
+    for p in orc.gen_positions(61, 12, 10, 50):
+        pos = np.array([p])
+        for depth in (3, 6):
+            want = orc.perft(int(p["black"]), int(p["white"]), int(p["to_move"]), depth, True)
+            assert mcts.perft(pos, depth, True) == want
