@@ -27,8 +27,11 @@
 #ifndef MCTS_EAST_F
 #define MCTS_EAST_F 1    // horizontal carry moves with IMAD shifts/adds
 #endif
-#ifndef MCTS_FLIP_WIDE
-#define MCTS_FLIP_WIDE 0 // flip carries with IMAD.WIDE instead of IADD3 pairs
+#ifndef MCTS_SPLIT
+#define MCTS_SPLIT 1     // vertical/diagonal move fills on 32-bit halves (one cross term per direction)
+#endif
+#ifndef MCTS_FLIP_K
+#define MCTS_FLIP_K 1    // flip carries from K = ~ray + first (saves the O | ~ray and 2 LOP3/direction)
 #endif
 
 namespace mcts_dev {
@@ -215,7 +218,7 @@ __device__ __forceinline__ u64 east_moves(u64 P, u64 M) {
 
 // One upward direction (+S, S in {7, 8, 9}) by a doubled-propagator fill: two
 // single steps cover a 2-disc run, two double steps (M2 = M & M<<S) extend it
-// to the 6-disc maximum. Left shifts only.
+// to the 6-disc maximum. Left shifts only (MCTS_SPLIT = 0 path).
 template <int S>
 __device__ __forceinline__ u64 up_moves(u64 P, u64 M) {
   const u64 M2 = M & (M << S);
@@ -226,6 +229,40 @@ __device__ __forceinline__ u64 up_moves(u64 P, u64 M) {
   return t << S;
 }
 
+// The same direction on 32-bit halves (rows 0-3 in lo, rows 4-7 in hi). An
+// upward run only ever moves from lo into hi, so lo is filled on its own
+// (three steps reach row 3 from row 0), then its top row crosses into hi once
+// — with P's top row, as the seed of the hi fill (three steps reach row 6 from
+// row 4) — instead of a funnel shift at every step of a 64-bit fill. All
+// left shifts are IMADs by 2^S (FMA pipe); the two cross terms are the only
+// shifts left on the ALU pipe. The landing squares t << S are or-ed into
+// (ml, mh).
+// One LOP3 with a fixed truth table (a = 0xF0, b = 0xCC, c = 0xAA). Written as
+// PTX so ptxas keeps the shared masks M in registers instead of re-fusing
+// O & kInner into every step (which costs a second LOP3 per step).
+template <u32 LUT>
+__device__ __forceinline__ u32 lop3(u32 a, u32 b, u32 c) {
+  u32 r;
+  asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(r) : "r"(a), "r"(b), "r"(c), "n"(LUT));
+  return r;
+}
+constexpr u32 kOrAnd = 0xF8;  // a | (b & c)
+constexpr u32 kAndOr = 0xA8;  // (a | b) & c
+
+template <int S>
+__device__ __forceinline__ void up_moves_split(u32 Pl, u32 Ph, u32 Ml, u32 Mh, u32& ml, u32& mh) {
+  const u32 p = c_pow2[S];
+  u32 tl = Ml & (Pl * p);
+  tl = lop3<kOrAnd>(tl, Ml, tl * p);
+  tl = lop3<kOrAnd>(tl, Ml, tl * p);
+  const u32 xp = Pl >> (32 - S), xt = tl >> (32 - S);
+  u32 th = lop3<kAndOr>(Ph * p + xp, xt, Mh);
+  th = lop3<kOrAnd>(th, Mh, th * p);
+  th = lop3<kOrAnd>(th, Mh, th * p);
+  ml |= tl * p;
+  mh |= th * p + xt;
+}
+
 // Legal moves. The four upward directions (+1 by carries, +7/+8/+9 by fills)
 // run on the board; the four downward ones run as upward directions of the
 // bit-reversed board rP/rO (square s -> 63 - s is the 180-degree rotation, so
@@ -233,6 +270,17 @@ __device__ __forceinline__ u64 up_moves(u64 P, u64 M) {
 // reuses rP/rO for the flips.
 __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
   const u64 M = O & kInner, rM = rO & kInner;
+#if MCTS_SPLIT
+  const u64 e = east_moves(P, M), re = east_moves(rP, rM);
+  u32 ml = (u32)e, mh = (u32)(e >> 32), rl = (u32)re, rh = (u32)(re >> 32);
+  up_moves_split<8>((u32)P, (u32)(P >> 32), (u32)O, (u32)(O >> 32), ml, mh);
+  up_moves_split<7>((u32)P, (u32)(P >> 32), (u32)M, (u32)(M >> 32), ml, mh);
+  up_moves_split<9>((u32)P, (u32)(P >> 32), (u32)M, (u32)(M >> 32), ml, mh);
+  up_moves_split<8>((u32)rP, (u32)(rP >> 32), (u32)rO, (u32)(rO >> 32), rl, rh);
+  up_moves_split<7>((u32)rP, (u32)(rP >> 32), (u32)rM, (u32)(rM >> 32), rl, rh);
+  up_moves_split<9>((u32)rP, (u32)(rP >> 32), (u32)rM, (u32)(rM >> 32), rl, rh);
+  return (join32(ml, mh) | __brevll(join32(rl, rh))) & ~(P | O);
+#else
   u64 m = east_moves(P, M);
   m |= up_moves<8>(P, O);
   m |= up_moves<7>(P, M);
@@ -242,6 +290,7 @@ __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
   r |= up_moves<7>(rP, rM);
   r |= up_moves<9>(rP, rM);
   return (m | __brevll(r)) & ~(P | O);
+#endif
 }
 
 // Upward ray masks (squares strictly beyond sq in direction +1, +8, +7, +9 up
@@ -261,7 +310,8 @@ __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
 }
 
 // Per-CTA shared table (u64 words): [0,256) ray masks rays[d*64 + sq],
-// [256,512) the ray's first square (0 at an edge), [512,768) a byte-select LUT:
+// [256,512) the carry addend of the ray (K = ~ray + first square, mod 2^64;
+// the first square alone when MCTS_FLIP_K = 0), [512,768) a byte-select LUT:
 // byte (k*256 + b) = index of the k-th set bit of the byte b.
 constexpr int kRayTable = 768;
 
@@ -270,7 +320,11 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
   for (int i = threadIdx.x; i < 256; i += blockDim.x) {
     const u64 m = ray_mask(i >> 6, i & 63);
     rays[i] = m;
+#if MCTS_FLIP_K
+    rays[256 + i] = ~m + (m & (0ULL - m));
+#else
     rays[256 + i] = m & (0ULL - m);
+#endif
     u64 packed = 0;  // LUT bytes 8i .. 8i+7
     for (int j = 0; j < 8; ++j) {
       const int e = 8 * i + j, k = e >> 8, b = e & 255;
@@ -283,23 +337,23 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
   }
 }
 
-// Flips along an upward ray by carry propagation: adding the ray's first square
-// to (O | ~m) carries through the contiguous opponent run (and through the
-// non-ray bits, all ones) and lands on the first non-opponent ray square.
-// run = ray squares that carried (~s & O & m); kept iff the landing square is P.
-__device__ __forceinline__ void up_flips(u64& f, u64 first, u64 P, u64 O, u64 m) {
-  const u64 xo = O | ~m;
-#if MCTS_FLIP_WIDE
-  // xo + first on the FMA pipe: IMAD for the high words, then one IMAD.WIDE
-  // (xo_lo * 1 + {first_lo, xo_hi + first_hi}) carries the low word into them.
-  const u32 one = c_pow2[0];
-  const u32 hi = (u32)(first >> 32) * one + (u32)(xo >> 32);
-  u64 s;
-  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(s) : "r"((u32)xo), "r"(one), "l"(join32((u32)first, hi)));
+// Flips along an upward ray m by carry propagation: adding the ray's first
+// square to (O | ~m) carries through the contiguous opponent run (and through
+// the non-ray bits, all ones) and lands on the first non-opponent ray square.
+// run = ray squares that carried (~s & O & m); kept iff the landing square
+// s & m & P is non-empty. With MCTS_FLIP_K the sum is formed as (O & m) + K,
+// K = ~m + first (O & m and ~m share no bits, so O | ~m = (O & m) + ~m): one
+// LOP3 per half for O & m, and the run update f | (~s & Om) is one 3-input
+// LOP3 per half.
+__device__ __forceinline__ void up_flips(u64& f, u64 k, u64 P, u64 O, u64 m) {
+#if MCTS_FLIP_K
+  const u64 Om = O & m;
+  const u64 s = Om + k;
+  if (s & m & P) f |= ~s & Om;
 #else
-  const u64 s = xo + first;
-#endif
+  const u64 s = (O | ~m) + k;
   if (s & m & P) f |= ~s & O & m;
+#endif
 }
 
 // All 8 directions: the 4 upward ones on the board, the 4 downward ones as

@@ -11,7 +11,11 @@ VARIANTS = {
     "no_upd_f": ["MCTS_UPD_F=0"],
     "no_east_f": ["MCTS_EAST_F=0"],
     "t128": ["MCTS_PLAYOUT_THREADS=128"],
-    "flip_wide": ["MCTS_FLIP_WIDE=1"],
+    "flip_k0": ["MCTS_FLIP_K=0"],
+    "split0": ["MCTS_SPLIT=0"],
+    "minb4": ["MCTS_PLAYOUT_MINB=4"],
+    "minb5": ["MCTS_PLAYOUT_MINB=5"],
+    "t128b8": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=8"],
 }
 
 if __name__ == "__main__":

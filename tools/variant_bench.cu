@@ -57,10 +57,15 @@ int main(int argc, char** argv) {
     }
     float sum = 0, best = 1e9;
     for (float t : ms) { sum += t; if (t < best) best = t; }
-    mcts_wdl w0;
-    cudaMemcpy(&w0, d_out, sizeof(w0), cudaMemcpyDeviceToHost);
-    printf("%-60s mean %.4f ms  best %.4f ms  %.3e playouts/s  leaf0 %u/%u/%u\n", argv[a], sum / ms.size(), best,
-           n * (double)per / (sum / ms.size() / 1e3), w0.wins, w0.draws, w0.losses);
+    // Checksum of every leaf's W/D/L (FNV-1a): variants must agree bit-exactly.
+    std::vector<mcts_wdl> w(n);
+    cudaMemcpy(w.data(), d_out, n * sizeof(mcts_wdl), cudaMemcpyDeviceToHost);
+    uint64_t hsh = 1469598103934665603ULL;
+    for (const mcts_wdl& x : w)
+      for (uint32_t v : {x.wins, x.draws, x.losses}) { hsh ^= v; hsh *= 1099511628211ULL; }
+    printf("%-60s mean %.4f ms  best %.4f ms  %.3e playouts/s  wdl-hash %016llx  leaf0 %u/%u/%u\n", argv[a],
+           sum / ms.size(), best, n * (double)per / (sum / ms.size() / 1e3), (unsigned long long)hsh, w[0].wins,
+           w[0].draws, w[0].losses);
     destroy(h);
   }
   return 0;
