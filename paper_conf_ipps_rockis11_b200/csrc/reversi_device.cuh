@@ -30,6 +30,12 @@
 #ifndef MCTS_SPLIT
 #define MCTS_SPLIT 1     // vertical/diagonal move fills on 32-bit halves (one cross term per direction)
 #endif
+#ifndef MCTS_FLIP_XY
+#define MCTS_FLIP_XY 1   // flips with one frame's rays on 32-bit words (see flips_hot_xy)
+#endif
+#ifndef MCTS_BIT_LUT
+#define MCTS_BIT_LUT 1   // 1 << sq from the shared table
+#endif
 #ifndef MCTS_FLIP_K
 #define MCTS_FLIP_K 1    // flip carries from K = ~ray + first (saves the O | ~ray and 2 LOP3/direction)
 #endif
@@ -312,8 +318,9 @@ __device__ __forceinline__ u64 ray_mask(int dir_index, int sq) {
 // Per-CTA shared table (u64 words): [0,256) ray masks rays[d*64 + sq],
 // [256,512) the carry addend of the ray (K = ~ray + first square, mod 2^64;
 // the first square alone when MCTS_FLIP_K = 0), [512,768) a byte-select LUT:
-// byte (k*256 + b) = index of the k-th set bit of the byte b.
-constexpr int kRayTable = 768;
+// byte (k*256 + b) = index of the k-th set bit of the byte b; [768,832) the
+// square bits 1 << sq (one LDS instead of two ALU-pipe shifts per ply).
+constexpr int kRayTable = 832;
 
 // Build the table (into global memory once per handle; CTAs copy it).
 __device__ __forceinline__ void fill_rays(u64* rays) {
@@ -334,6 +341,7 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
       packed |= (u64)pos << (8 * j);
     }
     rays[512 + i] = packed;
+    if (i < 64) rays[768 + i] = 1ULL << i;
   }
 }
 
@@ -374,6 +382,46 @@ __device__ __forceinline__ u64 flips_hot(int sq, u64 P, u64 O, u64 rP, u64 rO,
   return f | __brevll(g);
 }
 
+// One upward ray that lies inside a single 32-bit word (k = that word of K).
+// The 64-bit carry never leaves the ray's word, so the sum is a 32-bit add.
+__device__ __forceinline__ void up_flips32(u32& f, u32 k, u32 P, u32 O, u32 m) {
+  const u32 Om = O & m;
+  const u32 s = add_f(Om, k);
+  if (s & m & P) f |= ~s & Om;
+}
+
+// flips_hot with the rays split by half: of the two frames (board at sq, reversed
+// board at 63 - sq) exactly one puts the move in the hi word, and all four
+// upward rays from a hi-word square stay in the hi word (32-bit ops); the
+// other frame's square is in the lo word, where the +1 ray stays in the lo
+// word and only the +8/+7/+9 rays need 64-bit carries. The frames are chosen
+// per lane with selects (no divergence) and the result mapped back to the board.
+__device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO,
+                                            const u64* __restrict__ rays) {
+  const bool hx = sq >= 32;
+  const int xs = hx ? sq : 63 - sq, ys = 63 - xs;
+  const u32 XP = hx ? (u32)(P >> 32) : (u32)(rP >> 32);
+  const u32 XO = hx ? (u32)(O >> 32) : (u32)(rO >> 32);
+  const u64 YP = hx ? rP : P, YO = hx ? rO : O;
+  const u32* r32 = reinterpret_cast<const u32*>(rays);
+  u32 fx = 0;
+  up_flips32(fx, r32[2 * (256 + xs) + 1], XP, XO, r32[2 * xs + 1]);
+  up_flips32(fx, r32[2 * (320 + xs) + 1], XP, XO, r32[2 * (64 + xs) + 1]);
+  up_flips32(fx, r32[2 * (384 + xs) + 1], XP, XO, r32[2 * (128 + xs) + 1]);
+  up_flips32(fx, r32[2 * (448 + xs) + 1], XP, XO, r32[2 * (192 + xs) + 1]);
+  u32 fe = 0;
+  up_flips32(fe, r32[2 * (256 + ys)], (u32)YP, (u32)YO, r32[2 * ys]);
+  u64 fy = fe;
+  up_flips(fy, rays[320 + ys], YP, YO, rays[64 + ys]);
+  up_flips(fy, rays[384 + ys], YP, YO, rays[128 + ys]);
+  up_flips(fy, rays[448 + ys], YP, YO, rays[192 + ys]);
+  // Back to board coordinates: brev maps the other frame's word w to word 1-w.
+  const u32 yl = (u32)fy, yh = (u32)(fy >> 32);
+  const u32 lo = hx ? __brev(yh) : (__brev(fx) | yl);
+  const u32 hi = hx ? (fx | __brev(yl)) : yh;
+  return join32(lo, hi);
+}
+
 // k-th set bit: three popc levels down to a byte, then the byte-select LUT.
 __device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char* __restrict__ lut) {
   u32 lo = (u32)m, hi = (u32)(m >> 32);
@@ -399,8 +447,16 @@ __device__ __forceinline__ bool ply(u64& P, u64& O, PlayoutRng& rng, const u64* 
 #else
   const int sq = kth_set_bit(moves, k);
 #endif
+#if MCTS_FLIP_XY
+  const u64 f = flips_hot_xy(sq, P, O, rP, rO, rays);
+#else
   const u64 f = flips_hot(sq, P, O, rP, rO, rays);
+#endif
+#if MCTS_BIT_LUT
+  P = or_disjoint(P, or_disjoint(f, rays[768 + sq]));
+#else
   P = or_disjoint(P, or_disjoint(f, 1ULL << sq));
+#endif
   O = andnot_subset(O, f);
   return true;
 }

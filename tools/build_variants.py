@@ -14,8 +14,8 @@ VARIANTS = {
     "flip_k0": ["MCTS_FLIP_K=0"],
     "split0": ["MCTS_SPLIT=0"],
     "minb4": ["MCTS_PLAYOUT_MINB=4"],
-    "minb5": ["MCTS_PLAYOUT_MINB=5"],
-    "t128b8": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=8"],
+    "bitlut0": ["MCTS_BIT_LUT=0"],
+    "xy0": ["MCTS_FLIP_XY=0"],
 }
 
 if __name__ == "__main__":
