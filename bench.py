@@ -32,10 +32,27 @@ PLAYOUT_SEED = 2
 SEARCH_TREES, SEARCH_THREADS, SEARCH_MS = 1184, 128, 500.0
 LEAF_THREADS = 16384
 METRIC = "8x8 Reversi playouts/sec at 1/2/4/8 B200; win% vs CPU-oracle MCTS"
-# Algorithmic 32-bit integer operations per ply (one move decision) of the
-# shift-mask method, DESIGN.md §6 op model (movegen 2x8x24 incl. the final
-# shift + empty mask, flip 8x26, pick 30, Philox 96/4, loop 8).
+# SURVEY.md §8(d)'s a-priori estimate of 32-bit integer operations per ply of a
+# shift-mask implementation (movegen 2x8x24, flip 8x26, pick 30, Philox 96/4,
+# loop 8). The shipped loop needs far fewer, so the roofline's numerator is the
+# per-ply instruction count measured by ncu on the shipped kernel;
+# this figure is reported next to it as `survey_model` and is the fallback when
+# no capture is committed.
 ALG_OPS_PER_PLY = 440
+
+
+def ops_per_ply(kernel="playouts", plies_per_launch=None):
+    """(thread-instructions per ply, basis) for the roofline numerator: ncu
+    smsp__thread_inst_executed (= inst_executed x lanes active) of the committed
+    --set full capture of this kernel (profiles/latest_ncu.json), divided by the
+    plies of one launch of the same workload."""
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))[kernel]
+        plies = plies_per_launch or prof["plies_per_launch"]
+        return prof["thread_inst"] / plies, ("measured: ncu smsp__thread_inst_executed.sum / plies, "
+                                             f"committed capture of {kernel}_kernel (profiles/latest_ncu.json)")
+    except Exception:
+        return ALG_OPS_PER_PLY, "model: SURVEY.md 8(d) estimate (no committed capture)"
 
 
 def clocks_sampler(path):
@@ -513,8 +530,9 @@ def main():
             "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
-            # same per-ply op model as the headline roofline, per GPU
-            "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ALG_OPS_PER_PLY
+            # the playout kernel's measured instructions per ply (the search
+            # kernel's playouts run the same loop), per GPU
+            "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ops_per_ply("playouts")[0]
                              / integer_peak()[0],
         }
         log('ml = pkg.Mcts(')
@@ -543,14 +561,14 @@ def main():
     peak_ops, peak_basis, alu_peak = integer_peak()
     kern_s = kernel_ms / 1e3 / args.steps
     plies_per_launch = plies_local / args.steps
-    achieved = plies_per_launch * ALG_OPS_PER_PLY / kern_s
+    opp, opp_basis = ops_per_ply("playouts", plies_per_launch)
+    achieved = plies_per_launch * opp / kern_s
     traffic, ncu = None, None
     try:  # from the committed ncu --set full capture of this kernel (profiles/latest_ncu.json)
         prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))["playouts"]
         traffic = prof["dram_bytes_per_launch"]
         ncu = {k: prof.get(k) for k in ("alu_pipe_pct", "fmaheavy_pipe_pct", "issue_active_pct",
-                                        "lanes_active_per_inst", "thread_inst")}
-        ncu["thread_inst_per_ply"] = prof["thread_inst"] / plies_per_launch if prof.get("thread_inst") else None
+                                        "lanes_active_per_inst", "thread_inst", "duration_us")}
     except Exception:
         pass
     line = {
@@ -566,8 +584,10 @@ def main():
         "plies_per_s": plies_total / (t_ms / 1e3),
         "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak_ops / 1e9,
                      "unit": "Gop/s", "frac": achieved / peak_ops, "traffic": traffic,
-                     "ops_per_ply": ALG_OPS_PER_PLY, "plies_per_launch": plies_per_launch, "ncu": ncu,
-                     "peak_basis": peak_basis, "alu_pipe_peak": alu_peak / 1e9},
+                     "ops_per_ply": opp, "ops_basis": opp_basis, "plies_per_launch": plies_per_launch,
+                     "ncu": ncu, "peak_basis": peak_basis, "alu_pipe_peak": alu_peak / 1e9,
+                     "survey_model": {"ops_per_ply": ALG_OPS_PER_PLY,
+                                      "frac": plies_per_launch * ALG_OPS_PER_PLY / kern_s / peak_ops}},
         "e2e": {"value": e2e_value, "unit": "playouts/s",
                 "h2d_bytes_per_step": N_LEAVES * 24, "d2h_bytes_per_step": N_LEAVES * 12 + 8,
                 "api": "mcts_playouts (host buffers, pinned)"},

@@ -43,6 +43,12 @@ for k in ["playouts", "block_search", "leaf_search"]:
                  "duration_us": num("gpu__time_duration.sum"),
                  "thread_inst": float(d["smsp__inst_executed.sum"][0].replace(",", "")) *
                  float(d["smsp__thread_inst_executed_per_inst_executed.ratio"][0])}
+    if k == "playouts":  # the captured launch is one configs[1] batch (bench.py default workload)
+        try:
+            b = json.loads(open(os.path.join(ROOT, "gpurun_out", f"{tag}_bench.json")).read().splitlines()[-1])
+            latest[k]["plies_per_launch"] = b["roofline"]["plies_per_launch"]
+        except Exception:
+            latest[k]["plies_per_launch"] = 31433234.0  # configs[1], deterministic (bit-exact W/D/L)
 launch_csv = os.path.join(ROOT, "gpurun_out", f"{tag}_launches.csv")
 if os.path.exists(launch_csv):
     lines = open(launch_csv).read().splitlines()
