@@ -415,11 +415,11 @@ __device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO
   up_flips(fy, rays[320 + ys], YP, YO, rays[64 + ys]);
   up_flips(fy, rays[384 + ys], YP, YO, rays[128 + ys]);
   up_flips(fy, rays[448 + ys], YP, YO, rays[192 + ys]);
-  // Back to board coordinates: brev maps the other frame's word w to word 1-w.
-  const u32 yl = (u32)fy, yh = (u32)(fy >> 32);
-  const u32 lo = hx ? __brev(yh) : (__brev(fx) | yl);
-  const u32 hi = hx ? (fx | __brev(yl)) : yh;
-  return join32(lo, hi);
+  // Back to board coordinates: f = v | brev(u), u the reversed frame's flips
+  // and v the board frame's (brev maps word w of one frame to word 1-w).
+  const u64 u = hx ? fy : join32(0u, fx);
+  const u64 v = hx ? join32(0u, fx) : fy;
+  return v | __brevll(u);
 }
 
 // k-th set bit: three popc levels down to a byte, then the byte-select LUT.
