@@ -28,6 +28,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 N_LEAVES, N_PER_LEAF, GEN_SEED, LMIN, LMAX = 4096, 256, 2, 20, 40
+OPEN_LMIN, OPEN_LMAX = 0, 8  # the opening-phase batch
 PLAYOUT_SEED = 2
 SEARCH_TREES, SEARCH_THREADS, SEARCH_MS = 1184, 128, 500.0
 LEAF_THREADS = 16384
@@ -494,12 +495,41 @@ def main():
     barrier()
     e2e_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_s
 
+    log('# ---- opening-phase batch')
+    # ---- the same kernel on an opening-phase batch (L in [0, 8] random plies:
+    # the ~60-ply regime of playouts near the root), device-timed the same way
+    d_open = dev.gen_positions(m, GEN_SEED, N_LEAVES, OPEN_LMIN, OPEN_LMAX)
+    d_plies.zero_()
+    open_steps = max(3, args.steps // 4)
+    m.playouts_async(d_open.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, leaf_base,
+                     d_out.data_ptr(), 0, stream)
+    torch.cuda.synchronize()
+    barrier()
+    o_ms = 0.0
+    for _ in range(open_steps):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        m.playouts_async(d_open.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, leaf_base,
+                         d_out.data_ptr(), d_plies.data_ptr(), stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        o_ms += e0.elapsed_time(e1)
+    o_ms = max_over_ranks(o_ms)
+    o_plies = sum_over_ranks(int(d_plies.item()))
+    opening_batch = {
+        "workload": f"{N_LEAVES} synthetic opening-phase positions (seed {GEN_SEED}, "
+                    f"{OPEN_LMIN}-{OPEN_LMAX} random plies) x {N_PER_LEAF} playouts per GPU",
+        "playouts_per_s": world * open_steps * N_LEAVES * N_PER_LEAF / (o_ms / 1e3),
+        "plies_per_s": o_plies / (o_ms / 1e3), "ms_per_step": o_ms / open_steps,
+    }
+
     log('# ---- block-parallel search')
     # ---- block-parallel search (configs[2] shape) and leaf-parallel comparison
     # (configs[3]), time mode (or --search-iters for profiling), + root allreduce
     search = None
     leaf_search = None
-    launches = args.steps  # one playouts_kernel per timed step
+    launches = args.steps  # one playouts_kernel per timed step (the headline region)
 
     def run_search(handle, n_trees, threads, id_base):
         root = pkg.position(*pkg.OPENING)
@@ -593,7 +623,7 @@ def main():
                 "api": "mcts_playouts (host buffers, pinned)"},
         "gpu_launches": launches,
         "clocks": clocks,
-        "search": search, "leaf_search": leaf_search,
+        "opening_batch": opening_batch, "search": search, "leaf_search": leaf_search,
     }
     log('if not args.no_cpu and world =')
     if not args.no_cpu and world == 1:
