@@ -301,7 +301,7 @@ __global__ void stamp_kernel(u64* t0) { *t0 = globaltimer_ns(); }
 
 // ---------------------------------------------------------------------------
 // Perft (leaf count of the move tree to a given depth) with the hot-loop move
-// generator and flips (legal_moves_hot / flips_hot), to pin them directly to
+// generator and flips (legal_moves_hot / flips_loop), to pin them directly to
 // the north_star perft counts. Stage 1 (one thread) lists the frontier at
 // depth `split`; stage 2 runs one depth-first search per frontier node with an
 // explicit stack. A game-over node before the depth counts 1; a pass consumes
@@ -355,7 +355,7 @@ __device__ unsigned long long perft_dfs(u64 own, u64 opp, u32 depth, u32 pass_is
     if (f.moves == 0ULL) { --sp; continue; }
     const int sq = __ffsll((long long)f.moves) - 1;
     f.moves &= f.moves - 1;
-    const u64 fl = flips_hot(sq, f.own, f.opp, __brevll(f.own), __brevll(f.opp), rays);
+    const u64 fl = flips_loop(sq, f.own, f.opp, __brevll(f.own), __brevll(f.opp), rays);
     const u64 o = f.opp & ~fl, p = f.own | fl | (1ULL << sq);
     push(o, p, f.depth - 1);
   }

@@ -8,12 +8,14 @@
 // Two layers:
 //   * plain reference-style functions (legal_moves, flips, kth_set_bit) used by
 //     the tree code and the input generator, where speed does not matter;
-//   * the hot ply loop (legal_moves_hot, flips_hot, kth_set_bit_lut, ply,
-//     playout), shaped for the B200 integer pipes — see DESIGN.md §6: the loop
-//     is bound by the ALU pipe (LOP3/SHF/IADD3/SEL, 16 lanes/SMSP/clk), so work
-//     that can be done as plain 32-bit IMADs (FMA pipe) is, carries replace
-//     shift-fills where a ray is contiguous in bits, and every shift is a left
-//     shift (IMAD.SHL low word + one funnel SHF high word).
+//   * the hot ply loop (legal_moves_hot, flips_loop, kth_set_bit_lut, ply,
+//     playout), shaped for the B200 integer pipes — see DESIGN.md §5-§6: the
+//     loop is bound by the ALU pipe (LOP3/SHF/IADD3/SEL, 16 lanes/SMSP/clk), so
+//     it is written to need as few ALU-pipe instructions as possible: downward
+//     directions run as upward ones on the bit-reversed board (left shifts are
+//     IMADs by 2^S on the FMA pipe), vertical/diagonal move fills run on 32-bit
+//     words with one cross term, horizontal moves and all flips use carries,
+//     and the flips of the frame whose move lies in the hi word are 32-bit.
 #pragma once
 #include <cstdint>
 
@@ -29,6 +31,12 @@
 #endif
 #ifndef MCTS_SPLIT
 #define MCTS_SPLIT 1     // vertical/diagonal move fills on 32-bit halves (one cross term per direction)
+#endif
+#ifndef MCTS_FLIP_WIDE
+#define MCTS_FLIP_WIDE 0 // 64-bit flip carries as IMAD + IMAD.WIDE instead of IADD3 + IMAD.X
+#endif
+#ifndef MCTS_SHR_F
+#define MCTS_SHR_F 0     // cross-word right shifts of the split fills as IMAD.HI
 #endif
 #ifndef MCTS_FLIP_XY
 #define MCTS_FLIP_XY 1   // flips with one frame's rays on 32-bit words (see flips_hot_xy)
@@ -261,7 +269,11 @@ __device__ __forceinline__ void up_moves_split(u32 Pl, u32 Ph, u32 Ml, u32 Mh, u
   u32 tl = Ml & (Pl * p);
   tl = lop3<kOrAnd>(tl, Ml, tl * p);
   tl = lop3<kOrAnd>(tl, Ml, tl * p);
+#if MCTS_SHR_F
+  const u32 xp = __umulhi(Pl, p), xt = __umulhi(tl, p);  // >> (32 - S) as IMAD.HI (FMA pipe)
+#else
   const u32 xp = Pl >> (32 - S), xt = tl >> (32 - S);
+#endif
   u32 th = lop3<kAndOr>(Ph * p + xp, xt, Mh);
   th = lop3<kOrAnd>(th, Mh, th * p);
   th = lop3<kOrAnd>(th, Mh, th * p);
@@ -356,7 +368,15 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
 __device__ __forceinline__ void up_flips(u64& f, u64 k, u64 P, u64 O, u64 m) {
 #if MCTS_FLIP_K
   const u64 Om = O & m;
+#if MCTS_FLIP_WIDE
+  // Om + k on the FMA pipe: IMAD for the high words, then one IMAD.WIDE
+  // (Om_lo * 1 + {k_lo, hi}) carries the low word into them.
+  const u32 hi = add_f((u32)(Om >> 32), (u32)(k >> 32));
+  u64 s;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(s) : "r"((u32)Om), "r"(c_pow2[0]), "l"(join32((u32)k, hi)));
+#else
   const u64 s = Om + k;
+#endif
   if (s & m & P) f |= ~s & Om;
 #else
   const u64 s = (O | ~m) + k;
@@ -422,6 +442,16 @@ __device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO
   return v | __brevll(u);
 }
 
+// The flips the ply loop uses (and the device perft pins).
+__device__ __forceinline__ u64 flips_loop(int sq, u64 P, u64 O, u64 rP, u64 rO,
+                                          const u64* __restrict__ rays) {
+#if MCTS_FLIP_XY
+  return flips_hot_xy(sq, P, O, rP, rO, rays);
+#else
+  return flips_hot(sq, P, O, rP, rO, rays);
+#endif
+}
+
 // k-th set bit: three popc levels down to a byte, then the byte-select LUT.
 __device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char* __restrict__ lut) {
   u32 lo = (u32)m, hi = (u32)(m >> 32);
@@ -447,11 +477,7 @@ __device__ __forceinline__ bool ply(u64& P, u64& O, PlayoutRng& rng, const u64* 
 #else
   const int sq = kth_set_bit(moves, k);
 #endif
-#if MCTS_FLIP_XY
-  const u64 f = flips_hot_xy(sq, P, O, rP, rO, rays);
-#else
-  const u64 f = flips_hot(sq, P, O, rP, rO, rays);
-#endif
+  const u64 f = flips_loop(sq, P, O, rP, rO, rays);
 #if MCTS_BIT_LUT
   P = or_disjoint(P, or_disjoint(f, rays[768 + sq]));
 #else

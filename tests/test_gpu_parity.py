@@ -213,6 +213,31 @@ def test_search_leaf_config3_shape(mcts_leaf, orc):
     _cmp_search(res, ostats, obest)
 
 
+@pytest.mark.parametrize("seed,lmin,lmax,threads,iters", [
+    (21, 40, 50, 128, 20),    # late game: passes inside playouts (lane pairs stay in lockstep)
+    (22, 0, 4, 256, 6),       # opening phase: ~60-ply playouts
+])
+def test_search_leaf_bit_exact_late_and_opening(mcts_leaf, orc, seed, lmin, lmax, threads, iters):
+    root = orc.gen_positions(seed, 1, lmin, lmax)
+    res = mcts_leaf.search(root, iterations=iters, n_trees=1, threads_per_tree=threads, seed=seed)
+    ostats, obest, oplies = orc.uct_search(root, 1, threads, iters, seed)
+    _cmp_search(res, ostats, obest)
+    assert res["plies"] == oplies
+
+
+def test_search_leaf_terminal_and_pass_roots(mcts_leaf, orc):
+    full_black = (1 << 40) - 1
+    full_white = ((1 << 64) - 1) & ~full_black
+    res = mcts_leaf.search(orc.position(full_black, full_white, 0), iterations=3, n_trees=1,
+                           threads_per_tree=128, seed=1)
+    assert res["best_move"] == -1 and (res["stats"] == 0).all()
+    root = orc.position(0b11, 0b100, 1)
+    res = mcts_leaf.search(root, iterations=4, n_trees=1, threads_per_tree=128, seed=2)
+    ostats, obest, oplies = orc.uct_search(root, 1, 128, 4, 2)
+    _cmp_search(res, ostats, obest)
+    assert res["best_move"] == 64 and res["plies"] == oplies
+
+
 def test_search_terminal_and_pass_roots(mcts, orc):
     full_black = (1 << 40) - 1
     full_white = ((1 << 64) - 1) & ~full_black
