@@ -32,12 +32,6 @@
 #ifndef MCTS_SPLIT
 #define MCTS_SPLIT 1     // vertical/diagonal move fills on 32-bit halves (one cross term per direction)
 #endif
-#ifndef MCTS_FLIP_WIDE
-#define MCTS_FLIP_WIDE 0 // 64-bit flip carries as IMAD + IMAD.WIDE instead of IADD3 + IMAD.X
-#endif
-#ifndef MCTS_SHR_F
-#define MCTS_SHR_F 0     // cross-word right shifts of the split fills as IMAD.HI
-#endif
 #ifndef MCTS_FLIP_XY
 #define MCTS_FLIP_XY 1   // flips with one frame's rays on 32-bit words (see flips_hot_xy)
 #endif
@@ -269,12 +263,9 @@ __device__ __forceinline__ void up_moves_split(u32 Pl, u32 Ph, u32 Ml, u32 Mh, u
   u32 tl = Ml & (Pl * p);
   tl = lop3<kOrAnd>(tl, Ml, tl * p);
   tl = lop3<kOrAnd>(tl, Ml, tl * p);
-#if MCTS_SHR_F
-  const u32 xp = __umulhi(Pl, p), xt = __umulhi(tl, p);  // >> (32 - S) as IMAD.HI (FMA pipe)
-#else
-  const u32 xp = Pl >> (32 - S), xt = tl >> (32 - S);
-#endif
-  u32 th = lop3<kAndOr>(Ph * p + xp, xt, Mh);
+  const u32 xt = tl >> (32 - S);
+  const u32 pf = (u32)((join32(Pl, Ph) << S) >> 32);  // one funnel SHF: Ph << S | Pl >> (32 - S)
+  u32 th = lop3<kAndOr>(pf, xt, Mh);
   th = lop3<kOrAnd>(th, Mh, th * p);
   th = lop3<kOrAnd>(th, Mh, th * p);
   ml |= tl * p;
@@ -368,15 +359,7 @@ __device__ __forceinline__ void fill_rays(u64* rays) {
 __device__ __forceinline__ void up_flips(u64& f, u64 k, u64 P, u64 O, u64 m) {
 #if MCTS_FLIP_K
   const u64 Om = O & m;
-#if MCTS_FLIP_WIDE
-  // Om + k on the FMA pipe: IMAD for the high words, then one IMAD.WIDE
-  // (Om_lo * 1 + {k_lo, hi}) carries the low word into them.
-  const u32 hi = add_f((u32)(Om >> 32), (u32)(k >> 32));
-  u64 s;
-  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(s) : "r"((u32)Om), "r"(c_pow2[0]), "l"(join32((u32)k, hi)));
-#else
   const u64 s = Om + k;
-#endif
   if (s & m & P) f |= ~s & Om;
 #else
   const u64 s = (O | ~m) + k;

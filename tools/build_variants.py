@@ -16,9 +16,6 @@ VARIANTS = {
     "minb4": ["MCTS_PLAYOUT_MINB=4"],
     "bitlut0": ["MCTS_BIT_LUT=0"],
     "xy0": ["MCTS_FLIP_XY=0"],
-    "shrf": ["MCTS_SHR_F=1"],
-    "wide": ["MCTS_FLIP_WIDE=1"],
-    "shrf_wide": ["MCTS_SHR_F=1", "MCTS_FLIP_WIDE=1"],
 }
 
 if __name__ == "__main__":
