@@ -210,7 +210,7 @@ def sweep_leg(args, local):
                       "points": points}), flush=True)
 
 
-def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag=""):
+def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", opp_move=None):
     """Games of the B200 searcher (gpu_move(black, white, to_move, seed) ->
     (move, playouts)) against the oracle's root-parallel CPU MCTS on
     `cpu_threads` host threads, alternating colours, equal time per move; the
@@ -237,6 +237,9 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag=""):
             if to_move == gpu_color:
                 mv, po = gpu_move(black, white, to_move, seed)
                 gpu_po.append(po)
+            elif opp_move is not None:  # another device searcher (--h2h)
+                mv, po = opp_move(black, white, to_move, seed + 500)
+                cpu_po.append(po)
             else:
                 st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cpu_threads, move_ms, seed)
                 cpu_po.append(int(st[195]))
@@ -266,6 +269,40 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag=""):
             "gpu_playouts_per_move": float(np.mean(gpu_po)) if gpu_po else None,
             "cpu_playouts_per_move": float(np.mean(cpu_po)) if cpu_po else None,
             "wall_s": time.time() - t_start}
+
+
+def h2h_leg(args, local):
+    """configs[3] head-to-head: the block-parallel searcher
+    (configs[2], 1184 trees x 128 threads) against the paper's leaf-parallel
+    scheme (1 tree x 16384 threads per leaf batch) on the same GPU at equal wall
+    time per move, alternating colours. "gpu" in the result = the block side."""
+    import torch
+    import paper_conf_ipps_rockis11_b200 as pkg
+    torch.cuda.set_device(local)
+    stream = torch.cuda.current_stream()
+    st = torch.zeros(198, dtype=torch.int64, device="cuda")
+    hb = pkg.Mcts(c_uct=args.c_uct, scheme="block", device=local)
+    hl = pkg.Mcts(c_uct=args.c_uct, scheme="leaf", device=local)
+
+    def mover(h, n_trees, threads):
+        def move(black, white, to_move, seed):
+            h.search_async(pkg.position(black, white, to_move), 0, args.move_ms, n_trees, threads, seed, 0,
+                           st.data_ptr(), stream)
+            torch.cuda.synchronize()
+            x = st.cpu().numpy()
+            return pkg.best_move(x), int(x[195])
+        return move
+
+    r = play_match(mover(hb, SEARCH_TREES, SEARCH_THREADS), 0, args.selfplay, args.move_ms, tag="h2h",
+                   opp_move=mover(hl, 1, LEAF_THREADS))
+    r["block_playouts_per_move"] = r.pop("gpu_playouts_per_move")
+    r["leaf_playouts_per_move"] = r.pop("cpu_playouts_per_move")
+    print(json.dumps({"metric": "win% of block parallelism vs leaf parallelism (equal wall time per move)",
+                      "value": r["win_pct"], "unit": "%", "n_gpus": 1,
+                      "config": {"block": f"configs[2]: {SEARCH_TREES} trees x {SEARCH_THREADS} threads",
+                                 "leaf": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch",
+                                 "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct}, **r}),
+          flush=True)
 
 
 def selfplay_leg(args, world, rank, local):
@@ -388,6 +425,8 @@ def main():
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
+    ap.add_argument("--h2h", action="store_true",
+                    help="with --selfplay: block (configs[2]) vs leaf (configs[3]) head-to-head on one GPU")
     ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
     ap.add_argument("--sweep-games", type=int, default=0,
@@ -404,6 +443,8 @@ def main():
         local = 0
     if args.impl == "reference":
         return reference_arm(args, rank)
+    if args.selfplay and args.h2h:
+        return h2h_leg(args, local) if rank == 0 else None
     if args.selfplay:
         return selfplay_leg(args, world, rank, local)
     if args.sweep:

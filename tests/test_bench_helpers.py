@@ -30,3 +30,47 @@ def test_integer_peak_uses_measured_file():
     assert "measured" in basis
     # the measured mixed rate cannot exceed the issue-slot count at the max clock
     assert peak <= 148 * 4 * 32 * 1965e6 * 1.001
+
+
+def test_play_match_two_device_players_bookkeeping():
+    """play_match with opp_move (the --h2h leg) on two deterministic host movers:
+    the lowest-index legal move vs the highest. Colours alternate, so the two
+    games are mirror matches; results, disc differences and per-move counts
+    must be consistent with a replay under the oracle's rules."""
+    import oracle
+
+    def lowest(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        m = oracle.legal(own, opp)
+        return (m & -m).bit_length() - 1, 1
+
+    def highest(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        return oracle.legal(own, opp).bit_length() - 1, 2
+
+    r = bench.play_match(lowest, 0, 2, 1.0, opp_move=highest)
+    assert r["games"] == 2 and sum(r["results"].values()) == 2
+    assert r["gpu_playouts_per_move"] == 1 and r["cpu_playouts_per_move"] == 2
+
+    def replay(first_black):  # disc difference of `lowest` in one game
+        black, white, to_move = oracle.OPENING_BLACK, oracle.OPENING_WHITE, 0
+        while True:
+            own, opp = (black, white) if to_move == 0 else (white, black)
+            if oracle.legal(own, opp) == 0:
+                if oracle.legal(opp, own) == 0:
+                    break
+                to_move ^= 1
+                continue
+            lo_turn = (to_move == 0) == first_black
+            mv = (lowest if lo_turn else highest)(black, white, to_move, 0)[0]
+            f = oracle.flips(own, opp, mv)
+            own, opp = own | f | (1 << mv), opp & ~f
+            black, white = (own, opp) if to_move == 0 else (opp, own)
+            to_move ^= 1
+        d = bin(black).count("1") - bin(white).count("1")
+        return d if first_black else -d
+
+    want = [replay(True), replay(False)]
+    assert r["mean_disc_diff"] == sum(want) / 2
+    assert r["results"]["W"] == sum(d > 0 for d in want)
+    assert r["point_diff_per_step"][-1] == sum(want) / 2
