@@ -32,6 +32,12 @@ OPEN_LMIN, OPEN_LMAX = 0, 8  # the opening-phase batch
 PLAYOUT_SEED = 2
 SEARCH_TREES, SEARCH_THREADS, SEARCH_MS = 1184, 128, 500.0
 LEAF_THREADS = 16384
+# (n_trees, threads_per_tree) of each scheme's searcher; for "tree" n_trees is
+# the number of worker CTAs sharing one tree (NEXT-4)
+SCHEME_SHAPE = {"block": (SEARCH_TREES, SEARCH_THREADS), "leaf": (1, LEAF_THREADS),
+                "tree": (SEARCH_TREES, SEARCH_THREADS)}
+SCHEME_DESC = {"block": "configs[2] block-parallel", "leaf": "configs[3] leaf-parallel",
+               "tree": "NEXT-4 tree-parallel (one shared tree)"}
 METRIC = "8x8 Reversi playouts/sec at 1/2/4/8 B200; win% vs CPU-oracle MCTS"
 # SURVEY.md §8(d)'s a-priori estimate of 32-bit integer operations per ply of a
 # shift-mask implementation (movegen 2x8x24, flip 8x26, pick 30, Philox 96/4,
@@ -272,17 +278,20 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
 
 
 def h2h_leg(args, local):
-    """configs[3] head-to-head: the block-parallel searcher
+    """Head-to-head of two device searchers on the same GPU at equal wall time
+    per move, alternating colours (--h2h-schemes A,B; "gpu" in the result = A).
+    Default block,leaf = SURVEY.md 8(d) c3: the block-parallel searcher
     (configs[2], 1184 trees x 128 threads) against the paper's leaf-parallel
-    scheme (1 tree x 16384 threads per leaf batch) on the same GPU at equal wall
-    time per move, alternating colours. "gpu" in the result = the block side."""
+    scheme (1 tree x 16384 threads per leaf batch); tree,block pits the NEXT-4
+    shared tree (1184 workers x 128 threads) against configs[2]."""
     import torch
     import paper_conf_ipps_rockis11_b200 as pkg
     torch.cuda.set_device(local)
     stream = torch.cuda.current_stream()
     st = torch.zeros(198, dtype=torch.int64, device="cuda")
-    hb = pkg.Mcts(c_uct=args.c_uct, scheme="block", device=local)
-    hl = pkg.Mcts(c_uct=args.c_uct, scheme="leaf", device=local)
+    a, b = args.h2h_schemes.split(",")
+    ha = pkg.Mcts(c_uct=args.c_uct, scheme=a, device=local)
+    hb = pkg.Mcts(c_uct=args.c_uct, scheme=b, device=local)
 
     def mover(h, n_trees, threads):
         def move(black, white, to_move, seed):
@@ -293,15 +302,17 @@ def h2h_leg(args, local):
             return pkg.best_move(x), int(x[195])
         return move
 
-    r = play_match(mover(hb, SEARCH_TREES, SEARCH_THREADS), 0, args.selfplay, args.move_ms, tag="h2h",
-                   opp_move=mover(hl, 1, LEAF_THREADS))
-    r["block_playouts_per_move"] = r.pop("gpu_playouts_per_move")
-    r["leaf_playouts_per_move"] = r.pop("cpu_playouts_per_move")
-    print(json.dumps({"metric": "win% of block parallelism vs leaf parallelism (equal wall time per move)",
+    r = play_match(mover(ha, *SCHEME_SHAPE[a]), 0, args.selfplay, args.move_ms, tag="h2h",
+                   opp_move=mover(hb, *SCHEME_SHAPE[b]))
+    r[f"{a}_playouts_per_move"] = r.pop("gpu_playouts_per_move")
+    r[f"{b}_playouts_per_move"] = r.pop("cpu_playouts_per_move")
+    names = {"block": "block parallelism", "leaf": "leaf parallelism", "tree": "tree parallelism"}
+    shape = {k: f"{SCHEME_DESC[k]}: {v[0]} {'workers' if k == 'tree' else 'trees'} x {v[1]} threads"
+             for k, v in SCHEME_SHAPE.items()}
+    print(json.dumps({"metric": f"win% of {names[a]} vs {names[b]} (equal wall time per move)",
                       "value": r["win_pct"], "unit": "%", "n_gpus": 1,
-                      "config": {"block": f"configs[2]: {SEARCH_TREES} trees x {SEARCH_THREADS} threads",
-                                 "leaf": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch",
-                                 "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct}, **r}),
+                      "config": {a: shape[a], b: shape[b], "move_ms": args.move_ms, "colours": "alternating",
+                                 "C": args.c_uct}, **r}),
           flush=True)
 
 
@@ -324,8 +335,8 @@ def selfplay_leg(args, world, rank, local):
     hybrid = args.sp_scheme == "hybrid"
     if hybrid and world > 1:
         raise SystemExit("--sp-scheme hybrid is single-GPU")
-    scheme = "leaf" if args.sp_scheme == "leaf" else "block"
-    n_trees, threads = (SEARCH_TREES, SEARCH_THREADS) if scheme == "block" else (1, LEAF_THREADS)
+    scheme = {"leaf": "leaf", "tree": "tree"}.get(args.sp_scheme, "block")
+    n_trees, threads = SCHEME_SHAPE[scheme]
     m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
     stream = torch.cuda.current_stream()
     stats = torch.zeros(198, dtype=torch.int64, device="cuda")
@@ -365,8 +376,8 @@ def selfplay_leg(args, world, rank, local):
         return search(black, white, to_move, seed)
 
     cores = len(os.sched_getaffinity(0))
-    workload = (f"configs[{2 if scheme == 'block' else 3}] searcher ({n_trees} trees x {threads} "
-                f"threads per GPU, {args.sp_scheme}, {world} GPU(s))")
+    workload = (f"{SCHEME_DESC[scheme]} searcher ({n_trees} {'workers' if scheme == 'tree' else 'trees'} x "
+                f"{threads} threads per GPU, {args.sp_scheme}, {world} GPU(s))")
     if args.fig7:
         curves = []
         t = 1
@@ -421,12 +432,14 @@ def main():
     ap.add_argument("--selfplay", type=int, default=0,
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
-    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid"])
+    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid", "tree"])
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
     ap.add_argument("--h2h", action="store_true",
-                    help="with --selfplay: block (configs[2]) vs leaf (configs[3]) head-to-head on one GPU")
+                    help="with --selfplay: head-to-head of two device searchers on one GPU (--h2h-schemes)")
+    ap.add_argument("--h2h-schemes", default="block,leaf",
+                    help="A,B of block|leaf|tree (default block,leaf = configs[2] vs configs[3])")
     ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
     ap.add_argument("--sweep-games", type=int, default=0,
@@ -570,6 +583,7 @@ def main():
     # (configs[3]), time mode (or --search-iters for profiling), + root allreduce
     search = None
     leaf_search = None
+    tree_search = None
     launches = args.steps  # one playouts_kernel per timed step (the headline region)
 
     def run_search(handle, n_trees, threads, id_base):
@@ -616,6 +630,17 @@ def main():
             "best_move": int(pkg.best_move(lt)),
         }
         ml.close()
+        log('mt = pkg.Mcts(')
+        mt = pkg.Mcts(c_uct=1.0, scheme="tree", device=local)
+        tt, t_ms = run_search(mt, SEARCH_TREES, SEARCH_THREADS, rank)
+        tree_search = {
+            "workload": f"NEXT-4 tree parallelism: one shared tree, {SEARCH_TREES} workers x {SEARCH_THREADS} "
+                        f"threads per GPU, {mode}, opening root, C=1.0",
+            "playouts_per_s": float(tt[195]) / (t_ms / 1e3), "ms": t_ms,
+            "iterations": float(tt[196]) / world, "plies_per_s": float(tt[197]) / (t_ms / 1e3),
+            "best_move": int(pkg.best_move(tt)),
+        }
+        mt.close()
 
     log('if sampler is not None:')
     if sampler is not None:
@@ -665,6 +690,7 @@ def main():
         "gpu_launches": launches,
         "clocks": clocks,
         "opening_batch": opening_batch, "search": search, "leaf_search": leaf_search,
+        "tree_search": tree_search,
     }
     log('if not args.no_cpu and world =')
     if not args.no_cpu and world == 1:

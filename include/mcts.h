@@ -69,20 +69,28 @@ typedef struct {
 
 #define MCTS_BLOCK 0u /* block parallelism: one tree per CTA (L294-L311) */
 #define MCTS_LEAF 1u  /* leaf parallelism: one tree, the whole batch per leaf (L231-L237) */
+#define MCTS_TREE 2u  /* tree parallelism: every CTA on one shared tree with virtual loss
+                         (Chaslot et al.) */
+
+/* mcts_params.flags */
+#define MCTS_FLAG_CHECK_TREE 1u /* MCTS_TREE: after each search, check the tree invariants on the
+                                   device (vl = 0, k >= sum of children k (+1 below the root),
+                                   sum of k - children k = iterations); a violation makes
+                                   mcts_search return MCTS_E_CUDA */
 
 typedef struct {
   double c_uct;                /* UCB exploration constant C (L169); finite, >= 0; R1 default 1.0 */
-  uint32_t scheme;             /* MCTS_BLOCK or MCTS_LEAF */
-  uint32_t max_nodes_per_tree; /* time mode: node-slot pool per tree (0 = 65536) */
+  uint32_t scheme;             /* MCTS_BLOCK, MCTS_LEAF or MCTS_TREE */
+  uint32_t max_nodes_per_tree; /* time mode: node-slot pool per tree (0 = 65536; MCTS_TREE: 2^26) */
   int32_t device;              /* CUDA device ordinal */
-  uint32_t flags;              /* reserved, 0 */
+  uint32_t flags;              /* 0 or MCTS_FLAG_CHECK_TREE; other bits: INVALID_ARGUMENT */
 } mcts_params;
 
 /* Exactly one of iterations / time_ms is non-zero. Iteration mode is
  * deterministic and bit-exact to the oracle; time mode (a %globaltimer
  * deadline per search) is not reproducible. */
 typedef struct {
-  uint64_t iterations; /* UCT iterations per tree */
+  uint64_t iterations; /* UCT iterations per tree (MCTS_TREE: in total over the workers) */
   double time_ms;      /* wall-clock budget of the search kernel */
 } mcts_budget;
 
@@ -146,6 +154,13 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
  *               per iteration per tree (L186-L195, L294-L311).
  *   MCTS_LEAF:  n_trees must be 1; threads_per_tree (multiple of 128, <= 65536)
  *               playouts from the same leaf per iteration (L231-L237).
+ *   MCTS_TREE:  ONE tree shared by n_trees workers (CTAs of threads_per_tree
+ *               threads, multiple of 32, <= 1024; n_trees <= 65536), virtual
+ *               loss in selection, a CAS per expansion. The
+ *               iteration budget is the total over the workers (<= 2^24);
+ *               c1 = a global iteration ticket. With n_trees == 1 the result
+ *               equals MCTS_BLOCK with one tree bit for bit; with more workers
+ *               it depends on timing (tree invariants: MCTS_FLAG_CHECK_TREE).
  * Playout streams: c0 = tree id, c1 = iteration, c2 = thread. root (host,
  * nullable = the create-time position). out (host) receives the root stats
  * summed over trees and the best move. Synchronous.

@@ -8,7 +8,7 @@ package is a thin ctypes binding plus torch plumbing (device memory, streams,
 torch.distributed for the one cross-GPU allreduce).
 """
 from ._native import (  # noqa: F401
-    EXPORTS, MCTS_BLOCK, MCTS_LEAF, POSITION_DTYPE, STATS_LEN, Mcts, MctsError, best_move, load,
+    EXPORTS, MCTS_BLOCK, MCTS_FLAG_CHECK_TREE, MCTS_LEAF, MCTS_TREE, POSITION_DTYPE, STATS_LEN, Mcts, MctsError, best_move, load,
     version,
 )
 from .positions import OPENING, opening, position, own_opp  # noqa: F401

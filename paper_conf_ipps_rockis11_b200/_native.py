@@ -17,7 +17,8 @@ POSITION_DTYPE = np.dtype(
 )
 WDL_DTYPE = np.dtype([("wins", "<u4"), ("draws", "<u4"), ("losses", "<u4")])
 STATS_LEN = 198
-MCTS_BLOCK, MCTS_LEAF = 0, 1
+MCTS_BLOCK, MCTS_LEAF, MCTS_TREE = 0, 1, 2
+MCTS_FLAG_CHECK_TREE = 1
 
 # every symbol include/mcts.h declares
 EXPORTS = (
@@ -124,10 +125,10 @@ class Mcts:
     """One library handle (mcts_create/mcts_destroy) bound to a device."""
 
     def __init__(self, position=None, c_uct: float = 1.0, scheme: str = "block",
-                 max_nodes_per_tree: int = 0, device: int = 0):
+                 max_nodes_per_tree: int = 0, device: int = 0, flags: int = 0):
         self.L = load()
-        sch = {"block": MCTS_BLOCK, "leaf": MCTS_LEAF}[scheme]
-        params = Params(c_uct, sch, max_nodes_per_tree, device, 0)
+        sch = {"block": MCTS_BLOCK, "leaf": MCTS_LEAF, "tree": MCTS_TREE}[scheme]
+        params = Params(c_uct, sch, max_nodes_per_tree, device, flags)
         h = ctypes.c_void_p()
         pp = ctypes.byref(_pos(position)) if position is not None else None
         st = self.L.mcts_create(pp, ctypes.byref(params), ctypes.byref(h))

@@ -5,6 +5,8 @@
 //                        (PAPER.md L294-L311), root merge fused at the end
 //   leaf_search_kernel   a12: leaf-parallel UCT, one tree, the whole grid
 //                        simulates from the same leaf
+//   tree_search_kernel   NEXT-4: tree parallelism, every CTA on one shared tree
+//                        with virtual loss (tree_parallel.cuh)
 //   ln_table_kernel      lnT[k] = RN(ln(k*unit)) for the UCB term (R9)
 //   gen_positions_kernel synthetic input recipe
 #pragma once
@@ -289,6 +291,12 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
+
+}  // namespace mcts_dev
+
+#include "tree_parallel.cuh"
+
+namespace mcts_dev {
 
 // ---------------------------------------------------------------------------
 __global__ void ln_table_kernel(double* __restrict__ out, u32 unit, u32 K) {

@@ -58,6 +58,7 @@ struct mcts_handle {
   unsigned long long* d_t0 = nullptr;
   int* d_error = nullptr;
   LeafSync* d_leafsync = nullptr;
+  TreeSync* d_treesync = nullptr;  // MCTS_TREE counters
   u64* d_rays = nullptr;      // ray table for the flip kernels (kRayTable u64)
   u32* d_work = nullptr;      // ring of playout work counters (one per launch)
   uint32_t work_slot = 0;
@@ -126,7 +127,7 @@ mcts_status ensure_lnT(mcts_handle* h, uint32_t unit, uint32_t K, cudaStream_t s
 // Carve a TreePool for n_trees * slot_cap slots out of one allocation.
 mcts_status ensure_pool(mcts_handle* h, uint32_t n_trees, uint32_t slot_cap, TreePool* T) {
   const size_t slots = (size_t)n_trees * slot_cap;
-  const size_t per = 3 * sizeof(u64) + 5 * sizeof(u32);
+  const size_t per = 3 * sizeof(u64) + 6 * sizeof(u32);
   const size_t bytes = slots * per + 8 * 256;
   if (bytes > (size_t)96 << 30)
     return fail(h, MCTS_E_OOM, "tree pool would exceed 96 GiB; lower iterations or max_nodes_per_tree");
@@ -142,6 +143,7 @@ mcts_status ensure_pool(mcts_handle* h, uint32_t n_trees, uint32_t slot_cap, Tre
   T->d = (u32*)take(slots * sizeof(u32));
   T->first = (u32*)take(slots * sizeof(u32));
   T->meta = (u32*)take(slots * sizeof(u32));
+  T->vl = (u32*)take(slots * sizeof(u32));
   T->slot_cap = slot_cap;
   return MCTS_OK;
 }
@@ -157,6 +159,48 @@ mcts_status launch_block(mcts_handle* h, uint32_t n_trees, uint32_t threads, con
                          const SearchArgs& a, cudaStream_t s) {
   block_search_kernel<MAXT, MINB><<<n_trees, threads, 0, s>>>(T, a);
   CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+template <int MAXT, int MINB>
+mcts_status launch_tree(mcts_handle* h, uint32_t workers, uint32_t threads, const TreePool& T,
+                        const SearchArgs& a, cudaStream_t s) {
+  tree_search_kernel<MAXT, MINB><<<workers, threads, 0, s>>>(T, a, h->d_treesync);
+  CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+// MCTS_TREE (tree_parallel.cuh): one shared tree, `workers` CTAs of `unit`
+// threads. Pool slots are cleared (meta = 0 marks unpublished), the root is
+// created by a one-thread kernel, then the search, the root merge and (with
+// MCTS_FLAG_CHECK_TREE) the invariant check, all in stream order.
+mcts_status tree_search_impl(mcts_handle* h, const mcts_position* rp, uint32_t workers, uint32_t unit,
+                             uint32_t slot_cap, SearchArgs a, cudaStream_t s) {
+  TreePool T;
+  mcts_status st = ensure_pool(h, 1, slot_cap, &T);
+  if (st) return st;
+  CK(h, cudaMemsetAsync(T.meta, 0, (size_t)slot_cap * sizeof(u32), s));
+  DevPosition root;
+  memcpy(&root, rp, sizeof(DevPosition));
+  tree_root_kernel<<<1, 1, 0, s>>>(T, h->d_treesync, root);
+  CK(h, cudaGetLastError());
+  if (a.budget_ns) {
+    stamp_kernel<<<1, 1, 0, s>>>(h->d_t0);
+    CK(h, cudaGetLastError());
+  }
+  if (unit <= 128) st = launch_tree<128, 8>(h, workers, unit, T, a, s);
+  else if (unit <= 256) st = launch_tree<256, 4>(h, workers, unit, T, a, s);
+  else if (unit <= 512) st = launch_tree<512, 2>(h, workers, unit, T, a, s);
+  else st = launch_tree<1024, 1>(h, workers, unit, T, a, s);
+  if (st) return st;
+  tree_merge_kernel<<<1, 32, 0, s>>>(T, unit, a.stats);
+  CK(h, cudaGetLastError());
+  if (h->params.flags & MCTS_FLAG_CHECK_TREE) {
+    tree_check_kernel<<<592, 256, 0, s>>>(T, h->d_treesync, unit, slot_cap, h->d_error);
+    CK(h, cudaGetLastError());
+    tree_check_total_kernel<<<1, 1, 0, s>>>(h->d_treesync, a.stats, h->d_error);
+    CK(h, cudaGetLastError());
+  }
   return MCTS_OK;
 }
 
@@ -176,18 +220,58 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
   if (n_trees == 0) return fail(h, MCTS_E_INVALID_ARGUMENT, "n_trees == 0");
   if (!d_stats) return fail(h, MCTS_E_INVALID_ARGUMENT, "d_stats == NULL");
   const bool leaf = h->params.scheme == MCTS_LEAF;
+  const bool tree = h->params.scheme == MCTS_TREE;
   if (leaf) {
     if (n_trees != 1) return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: n_trees must be 1");
     if (threads_per_tree == 0 || threads_per_tree % 128 || threads_per_tree > 65536)
       return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_LEAF: threads_per_tree must be a multiple of 128 in [128, 65536]");
   } else {
     if (threads_per_tree == 0 || threads_per_tree % 32 || threads_per_tree > 1024)
-      return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_BLOCK: threads_per_tree must be a multiple of 32 in [32, 1024] (PAPER.md L310-L311)");
+      return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_BLOCK / MCTS_TREE: threads_per_tree must be a multiple of 32 in [32, 1024] (PAPER.md L310-L311)");
   }
   const uint64_t unit = threads_per_tree;
   const uint64_t kmax_counts = 0xFFFFFFFFull / unit;  // node counters are u32
   uint64_t max_it;
   uint32_t slot_cap;
+  if (tree) {
+    // one shared tree: iterations are the total over all workers; the ln
+    // table also covers the workers' virtual visits (k + vl <= iterations + W)
+    if (n_trees > 65536) return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_TREE: n_trees (workers) must be <= 65536");
+    const uint64_t cap_it = kmax_counts < (1u << 24) ? kmax_counts : (1u << 24);
+    if (by_iter) {
+      if (budget.iterations > cap_it)
+        return fail(h, MCTS_E_INVALID_ARGUMENT, "MCTS_TREE: iterations * threads_per_tree must be < 2^32 and iterations <= 2^24");
+      max_it = budget.iterations;
+      // one node per iteration, each reserving <= 60 child slots: never full
+      const uint64_t need = 61 + max_it * 60;
+      slot_cap = (uint32_t)(need > 0x7FFFFFFFull ? 0x7FFFFFFFull : need);
+    } else {
+      max_it = cap_it;
+      slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree : (1u << 26);
+      if (slot_cap < 64) slot_cap = 64;
+    }
+    mcts_status st = check_device(h);
+    if (st) return st;
+    st = ensure_lnT(h, (uint32_t)unit, (uint32_t)(max_it + n_trees + 1), s);
+    if (st) return st;
+    CK(h, cudaMemsetAsync(d_stats, 0, MCTS_STATS_LEN * sizeof(long long), s));
+    CK(h, cudaMemsetAsync(h->d_error, 0, sizeof(int), s));
+    SearchArgs a;
+    memcpy(&a.root, rp, sizeof(DevPosition));
+    a.key = key_of(seed);
+    a.C = h->params.c_uct;
+    a.lnT = h->d_lnT;
+    a.stats = d_stats;
+    a.t0 = h->d_t0;
+    a.budget_ns = by_time ? (u64)llround(budget.time_ms * 1e6) : 0ULL;
+    if (by_time && a.budget_ns == 0) a.budget_ns = 1;
+    a.max_iterations = (u32)max_it;
+    a.tree_id_base = tree_id_base;
+    a.unit = (u32)unit;
+    a.error = h->d_error;
+    a.rays = h->d_rays;
+    return tree_search_impl(h, rp, n_trees, (uint32_t)unit, slot_cap, a, s);
+  }
   if (by_iter) {
     if (budget.iterations > kmax_counts || budget.iterations > (1u << 24))
       return fail(h, MCTS_E_INVALID_ARGUMENT, "iterations * threads_per_tree must be < 2^32 and iterations <= 2^24");
@@ -278,8 +362,10 @@ const char* mcts_last_error(const mcts_handle* h) {
 mcts_status mcts_create(const mcts_position* position, const mcts_params* params, mcts_handle** out) {
   if (!out || !params) return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "out / params is NULL");
   *out = nullptr;
-  if (params->scheme != MCTS_BLOCK && params->scheme != MCTS_LEAF)
-    return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->scheme must be MCTS_BLOCK or MCTS_LEAF");
+  if (params->scheme != MCTS_BLOCK && params->scheme != MCTS_LEAF && params->scheme != MCTS_TREE)
+    return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->scheme must be MCTS_BLOCK, MCTS_LEAF or MCTS_TREE");
+  if (params->flags & ~(uint32_t)MCTS_FLAG_CHECK_TREE)
+    return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->flags: unknown bits");
   if (!std::isfinite(params->c_uct) || params->c_uct < 0.0)
     return fail(nullptr, MCTS_E_INVALID_ARGUMENT, "params->c_uct must be finite and >= 0");
   if (position && !position_ok(*position))
@@ -306,6 +392,7 @@ mcts_status mcts_create(const mcts_position* position, const mcts_params* params
   if (e == cudaSuccess) e = cudaMalloc(&h->d_error, sizeof(int));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_plies, sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_leafsync, sizeof(LeafSync));
+  if (e == cudaSuccess) e = cudaMalloc(&h->d_treesync, sizeof(TreeSync));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_rays, kRayTable * sizeof(u64));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_work, kWorkSlots * sizeof(u32));
   if (e == cudaSuccess) {
@@ -340,6 +427,7 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_t0);
   cudaFree(h->d_error);
   cudaFree(h->d_leafsync);
+  cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
   if (h->stream) cudaStreamDestroy(h->stream);
@@ -433,6 +521,7 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   int herr = 0;
   CK(h, cudaMemcpyAsync(&herr, h->d_error, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CK(h, cudaStreamSynchronize(h->stream));
+  if (herr == 2) return fail(h, MCTS_E_CUDA, "MCTS_TREE: tree invariant check failed (MCTS_FLAG_CHECK_TREE)");
   if (herr) return fail(h, MCTS_E_CUDA, "search kernel reported an internal error");
   for (int i = 0; i < 65; ++i) {
     out->visits[i] = (uint64_t)hs[i];

@@ -29,6 +29,7 @@ struct TreePool {
   u32* d;      // drawn playouts
   u32* first;  // first child slot (tree-relative) or kNoChild
   u32* meta;   // nchild | limit << 8 | move << 16 | terminal << 24
+  u32* vl;     // virtual visits of in-flight workers (MCTS_TREE only, tree_parallel.cuh)
   u32 slot_cap;
 };
 
