@@ -171,7 +171,7 @@ mcts_status launch_tree(mcts_handle* h, uint32_t workers, uint32_t threads, cons
 }
 
 // MCTS_TREE (tree_parallel.cuh): one shared tree, `workers` CTAs of `unit`
-// threads. Pool slots are cleared (meta = 0 marks unpublished), the root is
+// threads. Pool fields are cleared (meta = 0 marks unpublished), the root is
 // created by a one-thread kernel, then the search, the root merge and (with
 // MCTS_FLAG_CHECK_TREE) the invariant check, all in stream order.
 mcts_status tree_search_impl(mcts_handle* h, const mcts_position* rp, uint32_t workers, uint32_t unit,
@@ -179,7 +179,13 @@ mcts_status tree_search_impl(mcts_handle* h, const mcts_position* rp, uint32_t w
   TreePool T;
   mcts_status st = ensure_pool(h, 1, slot_cap, &T);
   if (st) return st;
+  // cleared fields: a read racing a child's creation sees meta = 0 (skipped)
+  // or k = vl = w = 0 and first = kNoChild (tree_select_expand)
   CK(h, cudaMemsetAsync(T.meta, 0, (size_t)slot_cap * sizeof(u32), s));
+  CK(h, cudaMemsetAsync(T.k, 0, (size_t)slot_cap * sizeof(u32), s));
+  CK(h, cudaMemsetAsync(T.w, 0, (size_t)slot_cap * sizeof(u32), s));
+  CK(h, cudaMemsetAsync(T.vl, 0, (size_t)slot_cap * sizeof(u32), s));
+  CK(h, cudaMemsetAsync(T.first, 0xFF, (size_t)slot_cap * sizeof(u32), s));
   DevPosition root;
   memcpy(&root, rp, sizeof(DevPosition));
   tree_root_kernel<<<1, 1, 0, s>>>(T, h->d_treesync, root);

@@ -94,23 +94,33 @@ __global__ void tree_root_kernel(TreePool T, TreeSync* S, DevPosition root) {
 // Selection + expansion on the shared tree by one warp (see the header). The
 // path (shared) gets root..leaf; every node on it carries this worker's
 // virtual visit on return.
+//
+// One load round trip per level: the lanes read every child's (meta, k, vl, w,
+// first) together with relaxed loads, and the winner's values become the next
+// level's node state (its meta, first, and k + vl for the parent term) without
+// re-reading. A child read that races its creation sees either meta == 0
+// (skipped) or the cleared pool values (k = vl = w = 0, first = kNoChild:
+// the node is then simulated instead of descended; both harmless, W = 1 never
+// races). Boards are read after an acquire fence.
 __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSync* S, u32* path,
                                                        const double* __restrict__ lnT, u32 unit,
                                                        double C, int lane) {
   u32 v = 0;
   int depth = 0;
+  u32 meta = ld_acq(&T.meta[0]);
+  u32 first = ld_rlx(&T.first[0]);
+  u32 kp = ld_rlx(&T.k[0]) + ld_rlx(&T.vl[0]);  // read before our own virtual visit
+  __syncwarp();
   if (lane == 0) {
     path[0] = 0;
     atomicAdd(&T.vl[0], 1u);
   }
   for (;;) {
-    u32 meta = ld_acq(&T.meta[v]);
     if (meta_term(meta) || depth >= kMaxPath - 2) break;
-    const u32 first = ld_rlx(&T.first[v]);
-    if (first == kNoChild) break;  // pool was full when v was created: simulate from v
+    if (first == kNoChild) break;  // pool full when v was created (or a racing read): simulate from v
     // Expansion: claim the lowest-index untried move (one CAS on the counter).
     if (meta_nchild(meta) < meta_limit(meta)) {
-      u32 claimed = kNoChild;
+      u32 claimed = kNoChild, mnow = meta;
       if (lane == 0) {
         u32 m = meta;
         while (meta_nchild(m) < meta_limit(m)) {
@@ -118,7 +128,9 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
           if (old == m) { claimed = meta_nchild(m); break; }
           m = old;
         }
+        mnow = m;
         if (claimed != kNoChild) {
+          __threadfence();  // acquire: v's board was published before its meta
           const u64 own = __ldcg(&T.own[v]), opp = __ldcg(&T.opp[v]), lg = __ldcg(&T.legal[v]);
           const u32 c = first + claimed;
           if (lg == 0ULL) {
@@ -137,21 +149,24 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
         ++depth;
         break;
       }
-      meta = ld_acq(&T.meta[v]);  // fully claimed meanwhile: select among the children
+      meta = __shfl_sync(kFull, mnow, 0);  // fully claimed meanwhile: select among the children
     }
     // Selection: UCB over the published children with virtual visits.
     const u32 nch = meta_nchild(meta);
-    const u32 kp = ld_rlx(&T.k[v]) + ld_rlx(&T.vl[v]) - 1u;  // others below v
-    const double lnp = lnT[kp];
+    const double lnp = lnT[kp];  // parent count k + vl without our own virtual visit
     double best_u = -__longlong_as_double(0x7FF0000000000000LL);
-    u32 best_i = kNoChild;
+    u32 best_i = kNoChild, best_meta = 0, best_first = kNoChild, best_k = 0;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
       const u32 c = first + i;
-      if (ld_acq(&T.meta[c]) == 0u) continue;  // claimed, not yet published
-      u32 kc = ld_rlx(&T.k[c]) + ld_rlx(&T.vl[c]);
-      if (kc == 0u) kc = 1u;  // a racing backprop between the two reads
-      const double u = ucb_value(ld_rlx(&T.w[c]), kc, unit, lnp, C);
-      if (u > best_u || best_i == kNoChild) { best_u = u; best_i = i; }
+      const u32 mc = ld_rlx(&T.meta[c]);
+      const u32 kc = ld_rlx(&T.k[c]), vc = ld_rlx(&T.vl[c]), wc = ld_rlx(&T.w[c]);
+      const u32 fc = ld_rlx(&T.first[c]);
+      if (mc == 0u) continue;  // claimed, not yet published
+      const u32 kk = kc + vc;
+      const double u = ucb_value(wc, kk ? kk : 1u, unit, lnp, C);
+      if (u > best_u || best_i == kNoChild) {
+        best_u = u; best_i = i; best_meta = mc; best_first = fc; best_k = kk;
+      }
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
@@ -163,7 +178,11 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
       }
     }
     if (best_i == kNoChild) break;  // no child published yet: simulate from v
+    const int src = (int)(best_i & 31u);
     v = first + best_i;
+    meta = __shfl_sync(kFull, best_meta, src);
+    first = __shfl_sync(kFull, best_first, src);
+    kp = __shfl_sync(kFull, best_k, src);  // v's k + vl, read before our own virtual visit
     ++depth;
     if (lane == 0) {
       path[depth] = v;
@@ -171,6 +190,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
     }
   }
   __syncwarp();
+  __threadfence();  // acquire: the leaf's board was published before its meta
   LeafInfo L;
   L.own = __ldcg(&T.own[v]);
   L.opp = __ldcg(&T.opp[v]);
