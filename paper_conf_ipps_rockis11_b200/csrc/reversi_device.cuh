@@ -38,6 +38,18 @@
 #ifndef MCTS_BIT_LUT
 #define MCTS_BIT_LUT 1   // 1 << sq from the shared table
 #endif
+#ifndef MCTS_PICK_SHL
+#define MCTS_PICK_SHL 0  // k-th bit: popc of the low 16/8 bits as popc(x << 16/24) (IMAD) instead of a mask (LOP3)
+#endif
+#ifndef MCTS_MAPBACK3
+#define MCTS_MAPBACK3 0  // flips back to board coordinates with 3 BREV and 2 SEL per word pair instead of 2 BREV + 4 SEL
+#endif
+#ifndef MCTS_RM_BREV
+#define MCTS_RM_BREV 1   // reversed-board propagator mask as brev(O & inner) (XU) instead of rO & inner (ALU)
+#endif
+#ifndef MCTS_PRED_FLIP
+#define MCTS_PRED_FLIP 1 // 32-bit ray flips: the kept run or-ed in by one predicated LOP3
+#endif
 #ifndef MCTS_FLIP_K
 #define MCTS_FLIP_K 1    // flip carries from K = ~ray + first (saves the O | ~ray and 2 LOP3/direction)
 #endif
@@ -278,7 +290,11 @@ __device__ __forceinline__ void up_moves_split(u32 Pl, u32 Ph, u32 Ml, u32 Mh, u
 // -1/-7/-8/-9 become +1/+7/+8/+9 and the file masks are unchanged). The caller
 // reuses rP/rO for the flips.
 __device__ __forceinline__ u64 legal_moves_hot(u64 P, u64 O, u64 rP, u64 rO) {
+#if MCTS_RM_BREV
+  const u64 M = O & kInner, rM = __brevll(M);  // kInner is symmetric under bit reversal
+#else
   const u64 M = O & kInner, rM = rO & kInner;
+#endif
 #if MCTS_SPLIT
   const u64 e = east_moves(P, M), re = east_moves(rP, rM);
   u32 ml = (u32)e, mh = (u32)(e >> 32), rl = (u32)re, rh = (u32)(re >> 32);
@@ -390,7 +406,23 @@ __device__ __forceinline__ u64 flips_hot(int sq, u64 P, u64 O, u64 rP, u64 rO,
 __device__ __forceinline__ void up_flips32(u32& f, u32 k, u32 P, u32 O, u32 m) {
   const u32 Om = O & m;
   const u32 s = add_f(Om, k);
+#if MCTS_PRED_FLIP == 2
+  // no select: h = umulhi(L, 2^32 - 1) = L ? L - 1 : 0 for the landing bit L,
+  // and the kept run is ~s & m & h (the carried squares below L on the ray)
+  const u32 h = __umulhi(s & m & P, 0xFFFFFFFFu);
+  f |= ~s & m & h;
+#elif MCTS_PRED_FLIP
+  // f |= ~s & Om under the landing predicate as ONE predicated LOP3 (the C++
+  // form compiles to run LOP3 + SEL + a share of an OR-merge LOP3).
+  asm("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\t"
+      "lop3.b32 t, %1, %2, %3, 0x80;\n\t"   // s & m & P: the landing square
+      "setp.ne.u32 p, t, 0;\n\t"
+      "@p lop3.b32 %0, %0, %1, %4, 0xF2;\n\t"  // f | (~s & Om)
+      "}"
+      : "+r"(f) : "r"(s), "r"(m), "r"(P), "r"(Om));
+#else
   if (s & m & P) f |= ~s & Om;
+#endif
 }
 
 // flips_hot with the rays split by half: of the two frames (board at sq, reversed
@@ -420,9 +452,17 @@ __device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO
   up_flips(fy, rays[448 + ys], YP, YO, rays[192 + ys]);
   // Back to board coordinates: f = v | brev(u), u the reversed frame's flips
   // and v the board frame's (brev maps word w of one frame to word 1-w).
+#if MCTS_MAPBACK3
+  // hx: f = (fx << 32) | brev(fy); else f = fy | brev(fx << 32) = fy | brev(fx)
+  const u32 ylo = (u32)fy, yhi = (u32)(fy >> 32);
+  const u32 lo = hx ? __brev(yhi) : (ylo | __brev(fx));
+  const u32 hi = hx ? (fx | __brev(ylo)) : yhi;
+  return join32(lo, hi);
+#else
   const u64 u = hx ? fy : join32(0u, fx);
   const u64 v = hx ? join32(0u, fx) : fy;
   return v | __brevll(u);
+#endif
 }
 
 // The flips the ply loop uses (and the device perft pins).
@@ -443,8 +483,13 @@ __device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char
   u32 x = up ? hi : lo;
   k -= up ? c : 0u;
   int base = up ? 32 : 0;
+#if MCTS_PICK_SHL
+  c = __popc(x * c_pow2[16]); up = k >= c; x = up ? (x >> 16) : x; k -= up ? c : 0u; base += up ? 16 : 0;
+  c = __popc(x * c_pow2[24]); up = k >= c; x = up ? (x >> 8) : x;  k -= up ? c : 0u; base += up ? 8 : 0;
+#else
   c = __popc(x & 0xFFFFu); up = k >= c; x = up ? (x >> 16) : x; k -= up ? c : 0u; base += up ? 16 : 0;
   c = __popc(x & 0xFFu);   up = k >= c; x = up ? (x >> 8) : x;  k -= up ? c : 0u; base += up ? 8 : 0;
+#endif
   return base + lut[(k << 8) | (x & 0xFFu)];
 }
 

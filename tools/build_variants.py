@@ -16,6 +16,12 @@ VARIANTS = {
     "minb4": ["MCTS_PLAYOUT_MINB=4"],
     "bitlut0": ["MCTS_BIT_LUT=0"],
     "xy0": ["MCTS_FLIP_XY=0"],
+    "pred0": ["MCTS_PRED_FLIP=0"],
+    "pred2": ["MCTS_PRED_FLIP=2"],
+    "pshl": ["MCTS_PICK_SHL=1"],
+    "map3": ["MCTS_MAPBACK3=1"],
+    "rmb": ["MCTS_RM_BREV=1"],
+    "pr": ["MCTS_PICK_SHL=1", "MCTS_RM_BREV=1"],
 }
 
 if __name__ == "__main__":
