@@ -47,6 +47,15 @@
 #ifndef MCTS_RM_BREV
 #define MCTS_RM_BREV 1   // reversed-board propagator mask as brev(O & inner) (XU) instead of rO & inner (ALU)
 #endif
+#ifndef MCTS_HXP
+#define MCTS_HXP 1       // the flips' frame (square >= 32) taken from the pick's first popc level
+#endif
+#ifndef MCTS_NW
+#define MCTS_NW 1        // the ply counter doubles as the RNG word index (one increment per ply)
+#endif
+#ifndef MCTS_ZT
+#define MCTS_ZT 1        // no-move test as one 3-input LOP3 predicate on the two words
+#endif
 #ifndef MCTS_PRED_FLIP
 #define MCTS_PRED_FLIP 1 // 32-bit ray flips: the kept run or-ed in by one predicated LOP3
 #endif
@@ -178,6 +187,16 @@ struct PlayoutRng {
   __device__ __forceinline__ u32 next() {
     if ((w & 3u) == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, w >> 2), key);
     ++w;
+    const u32 r = buf.x;
+    buf.x = buf.y;
+    buf.y = buf.z;
+    buf.z = buf.w;
+    return r;
+  }
+  // The same stream with the word index kept by the caller (the playout's
+  // ply counter: one word per non-pass decision, so w == plies so far).
+  __device__ __forceinline__ u32 next_at(u32 n) {
+    if ((n & 3u) == 0u) buf = philox4x32_10(make_uint4(c0, c1, c2, n >> 2), key);
     const u32 r = buf.x;
     buf.x = buf.y;
     buf.y = buf.z;
@@ -432,8 +451,7 @@ __device__ __forceinline__ void up_flips32(u32& f, u32 k, u32 P, u32 O, u32 m) {
 // word and only the +8/+7/+9 rays need 64-bit carries. The frames are chosen
 // per lane with selects (no divergence) and the result mapped back to the board.
 __device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO,
-                                            const u64* __restrict__ rays) {
-  const bool hx = sq >= 32;
+                                            const u64* __restrict__ rays, bool hx) {
   const int xs = hx ? sq : 63 - sq, ys = 63 - xs;
   const u32 XP = hx ? (u32)(P >> 32) : (u32)(rP >> 32);
   const u32 XO = hx ? (u32)(O >> 32) : (u32)(rO >> 32);
@@ -469,17 +487,19 @@ __device__ __forceinline__ u64 flips_hot_xy(int sq, u64 P, u64 O, u64 rP, u64 rO
 __device__ __forceinline__ u64 flips_loop(int sq, u64 P, u64 O, u64 rP, u64 rO,
                                           const u64* __restrict__ rays) {
 #if MCTS_FLIP_XY
-  return flips_hot_xy(sq, P, O, rP, rO, rays);
+  return flips_hot_xy(sq, P, O, rP, rO, rays, sq >= 32);
 #else
   return flips_hot(sq, P, O, rP, rO, rays);
 #endif
 }
 
 // k-th set bit: three popc levels down to a byte, then the byte-select LUT.
-__device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char* __restrict__ lut) {
+__device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char* __restrict__ lut,
+                                               bool* in_hi = nullptr) {
   u32 lo = (u32)m, hi = (u32)(m >> 32);
   u32 c = __popc(lo);
   bool up = k >= c;
+  if (in_hi) *in_hi = up;  // the square is >= 32
   u32 x = up ? hi : lo;
   k -= up ? c : 0u;
   int base = up ? 32 : 0;
@@ -495,17 +515,31 @@ __device__ __forceinline__ int kth_set_bit_lut(u64 m, u32 k, const unsigned char
 
 // One decision for the side owning P: returns false if P has no move (a pass;
 // nothing changes, no RNG word consumed), else plays the uniformly random move.
-__device__ __forceinline__ bool ply(u64& P, u64& O, PlayoutRng& rng, const u64* __restrict__ rays) {
+__device__ __forceinline__ bool ply(u64& P, u64& O, PlayoutRng& rng, u32 n, const u64* __restrict__ rays) {
   const u64 rP = __brevll(P), rO = __brevll(O);
   const u64 moves = legal_moves_hot(P, O, rP, rO);
+#if MCTS_ZT
+  if (((u32)moves | (u32)(moves >> 32)) == 0u) return false;
+#else
   if (moves == 0ULL) return false;
+#endif
+#if MCTS_NW
+  const u32 k = __umulhi(rng.next_at(n), (u32)__popcll(moves));
+#else
   const u32 k = __umulhi(rng.next(), (u32)__popcll(moves));
+#endif
+#if MCTS_PICK_LUT && MCTS_FLIP_XY && MCTS_HXP
+  bool hx;  // the pick's first level already decided the half: the flips' frame
+  const int sq = kth_set_bit_lut(moves, k, reinterpret_cast<const unsigned char*>(rays + 512), &hx);
+  const u64 f = flips_hot_xy(sq, P, O, rP, rO, rays, hx);
+#else
 #if MCTS_PICK_LUT
   const int sq = kth_set_bit_lut(moves, k, reinterpret_cast<const unsigned char*>(rays + 512));
 #else
   const int sq = kth_set_bit(moves, k);
 #endif
   const u64 f = flips_loop(sq, P, O, rP, rO, rays);
+#endif
 #if MCTS_BIT_LUT
   P = or_disjoint(P, or_disjoint(f, rays[768 + sq]));
 #else
@@ -533,11 +567,11 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   const u32 empties = 64u - (u32)__popcll(me | op);
   for (;;) {
     if (n == empties) break;
-    if (ply(me, op, rng, rays)) { passed = false; ++n; }
+    if (ply(me, op, rng, n, rays)) { passed = false; ++n; }
     else if (passed) break;
     else passed = true;
     if (n == empties) break;
-    if (ply(op, me, rng, rays)) { passed = false; ++n; }
+    if (ply(op, me, rng, n, rays)) { passed = false; ++n; }
     else if (passed) break;
     else passed = true;
   }

@@ -21,7 +21,10 @@ VARIANTS = {
     "pshl": ["MCTS_PICK_SHL=1"],
     "map3": ["MCTS_MAPBACK3=1"],
     "rmb": ["MCTS_RM_BREV=1"],
-    "pr": ["MCTS_PICK_SHL=1", "MCTS_RM_BREV=1"],
+    "nw0": ["MCTS_NW=0"],
+    "zt0": ["MCTS_ZT=0"],
+    "hxp0": ["MCTS_HXP=0"],
+    "old3": ["MCTS_NW=0", "MCTS_ZT=0", "MCTS_HXP=0"],
 }
 
 if __name__ == "__main__":
