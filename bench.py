@@ -332,10 +332,10 @@ def selfplay_leg(args, world, rank, local):
     torch.cuda.set_device(local)
     if world > 1:
         init_dist(dist, torch, local)
-    hybrid = args.sp_scheme == "hybrid"
+    hybrid = args.sp_scheme in ("hybrid", "hybrid-tree")
     if hybrid and world > 1:
         raise SystemExit("--sp-scheme hybrid is single-GPU")
-    scheme = {"leaf": "leaf", "tree": "tree"}.get(args.sp_scheme, "block")
+    scheme = {"leaf": "leaf", "tree": "tree", "hybrid-tree": "tree"}.get(args.sp_scheme, "block")
     n_trees, threads = SCHEME_SHAPE[scheme]
     m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
     stream = torch.cuda.current_stream()
@@ -432,7 +432,7 @@ def main():
     ap.add_argument("--selfplay", type=int, default=0,
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
-    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid", "tree"])
+    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid", "tree", "hybrid-tree"])
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")

@@ -187,9 +187,10 @@ mcts_status mcts_search_async(mcts_handle* h, const mcts_position* root, mcts_bu
  * trees are summed (L199-L202) into out, the host trees' share alone into
  * out_cpu (nullable). Iteration mode: every GPU tree and every host tree runs
  * budget.iterations iterations (deterministic; host trees = the oracle's UCT
- * with unit 1). Time mode: both sides stop at time_ms. MCTS_BLOCK handles
- * only; errors as mcts_search plus INVALID_ARGUMENT for cpu_threads outside
- * [1, 1024]. Synchronous. */
+ * with unit 1). Time mode: both sides stop at time_ms. MCTS_BLOCK or
+ * MCTS_TREE handles (with MCTS_TREE the GPU part is the one shared tree of
+ * n_trees workers); errors as mcts_search plus INVALID_ARGUMENT for a
+ * MCTS_LEAF handle or cpu_threads outside [1, 1024]. Synchronous. */
 mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_budget budget,
                                uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
                                uint32_t cpu_threads, mcts_root_stats* out, mcts_root_stats* out_cpu);

@@ -560,7 +560,7 @@ mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_b
                                uint32_t cpu_threads, mcts_root_stats* out, mcts_root_stats* out_cpu) {
   if (!h) return MCTS_E_INVALID_ARGUMENT;
   if (!out) return fail(h, MCTS_E_INVALID_ARGUMENT, "out == NULL");
-  if (h->params.scheme != MCTS_BLOCK) return fail(h, MCTS_E_INVALID_ARGUMENT, "hybrid search needs MCTS_BLOCK");
+  if (h->params.scheme == MCTS_LEAF) return fail(h, MCTS_E_INVALID_ARGUMENT, "hybrid search needs MCTS_BLOCK or MCTS_TREE");
   if (cpu_threads == 0 || cpu_threads > 1024) return fail(h, MCTS_E_INVALID_ARGUMENT, "cpu_threads must be in [1, 1024]");
   const mcts_position* rp = root ? root : (h->has_position ? &h->position : nullptr);
   if (!rp) return fail(h, MCTS_E_INVALID_ARGUMENT, "no root position");
@@ -604,8 +604,12 @@ mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_b
   long long cs[MCTS_STATS_LEN];
   mcts_host::search(a, (int64_t*)cs);
   long long hs[MCTS_STATS_LEN];
+  int herr = 0;
   CK(h, cudaMemcpyAsync(hs, h->d_stats, sizeof(hs), cudaMemcpyDeviceToHost, h->stream));
+  CK(h, cudaMemcpyAsync(&herr, h->d_error, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CK(h, cudaStreamSynchronize(h->stream));
+  if (herr == 2) return fail(h, MCTS_E_CUDA, "MCTS_TREE: tree invariant check failed (MCTS_FLAG_CHECK_TREE)");
+  if (herr) return fail(h, MCTS_E_CUDA, "search kernel reported an internal error");
   if (out_cpu) fill_root_stats(cs, out_cpu);
   for (int i = 0; i < MCTS_STATS_LEN; ++i) hs[i] += cs[i];  // root sum over all trees (L199-L202)
   fill_root_stats(hs, out);

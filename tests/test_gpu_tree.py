@@ -129,3 +129,26 @@ def test_tree_argument_errors(orc):
     m.close()
     with pytest.raises(pkg.MctsError):
         pkg.Mcts(scheme="tree", device=0, flags=4)
+
+
+def test_tree_hybrid_iteration_mode(orc):
+    """NEXT-1 on top of NEXT-4: the shared tree (one worker: deterministic) plus
+    host trees, root sums merged — the oracle's two searches added up."""
+    m = _tree()
+    root = orc.gen_positions(42, 1, 20, 30)
+    res = m.search_hybrid(root, iterations=60, n_trees=1, threads_per_tree=64, seed=14, cpu_threads=3)
+    g, _, gp = orc.uct_search(root, 1, 64, 60, 14)
+    c, _, cp = orc.uct_search(root, 3, 1, 60, 14, tree_id_base=0x40000000)
+    merged = g + c
+    assert res["stats"][:197].tolist() == merged[:197].tolist()
+    assert res["plies"] == gp + cp
+    m.close()
+
+
+def test_tree_hybrid_time_mode(orc):
+    m = _tree()
+    root = orc.opening()
+    res = m.search_hybrid(root, time_ms=50.0, n_trees=592, threads_per_tree=128, seed=15, cpu_threads=4)
+    assert res["cpu"]["iterations"] > 0 and res["iterations"] > res["cpu"]["iterations"]
+    assert res["stats"][195] == (res["iterations"] - res["cpu"]["iterations"]) * 128 + res["cpu"]["iterations"]
+    m.close()
