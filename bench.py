@@ -586,10 +586,11 @@ def main():
     tree_search = None
     launches = args.steps  # one playouts_kernel per timed step (the headline region)
 
-    def run_search(handle, n_trees, threads, id_base):
+    def run_search(handle, n_trees, threads, id_base, it_scale=1):
+        # it_scale: the shared tree's iteration budget is a total over its workers
         root = pkg.position(*pkg.OPENING)
         st = torch.zeros(198, dtype=torch.int64, device="cuda")
-        it, ms = (args.search_iters, 0.0) if args.search_iters else (0, args.search_ms)
+        it, ms = (args.search_iters * it_scale, 0.0) if args.search_iters else (0, args.search_ms)
         handle.search_async(root, min(it, 2) if it else 0, 0.0 if it else 20.0, n_trees, threads,
                             1000, id_base, st.data_ptr(), stream)  # warm-up: pool + ln table
         torch.cuda.synchronize()
@@ -632,7 +633,7 @@ def main():
         ml.close()
         log('mt = pkg.Mcts(')
         mt = pkg.Mcts(c_uct=1.0, scheme="tree", device=local)
-        tt, t_ms = run_search(mt, SEARCH_TREES, SEARCH_THREADS, rank)
+        tt, t_ms = run_search(mt, SEARCH_TREES, SEARCH_THREADS, rank, it_scale=SEARCH_TREES)
         tree_search = {
             "workload": f"NEXT-4 tree parallelism: one shared tree, {SEARCH_TREES} workers x {SEARCH_THREADS} "
                         f"threads per GPU, {mode}, opening root, C=1.0",

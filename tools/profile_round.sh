@@ -14,3 +14,5 @@ timeout 400 ncu --set full --clock-control none --import-source on -k regex:bloc
   -o gpurun_out/${TAG}_block_search python bench.py --steps 1 --warmup 3 --no-cpu --search-iters 200 > /dev/null 2>&1; echo "ncu search rc=$?"
 timeout 400 ncu --set full --clock-control none --import-source on -k regex:leaf_search_kernel -s 1 -c 1 \
   -o gpurun_out/${TAG}_leaf_search python bench.py --steps 1 --warmup 3 --no-cpu --search-iters 200 > /dev/null 2>&1; echo "ncu leaf rc=$?"
+timeout 400 ncu --set full --clock-control none --import-source on -k regex:tree_search_kernel -s 1 -c 1 \
+  -o gpurun_out/${TAG}_tree_search python bench.py --steps 1 --warmup 3 --no-cpu --search-iters 200 > /dev/null 2>&1; echo "ncu tree rc=$?"

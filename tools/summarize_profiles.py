@@ -9,7 +9,7 @@ tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 out_dir = os.path.join(ROOT, "profiles")
 os.makedirs(out_dir, exist_ok=True)
 latest = {}
-for k in ["playouts", "block_search", "leaf_search"]:
+for k in ["playouts", "block_search", "leaf_search", "tree_search"]:
     rep = os.path.join(ROOT, "gpurun_out", f"{tag}_{k}.ncu-rep")
     if not os.path.exists(rep):
         continue
