@@ -169,18 +169,21 @@ def cpu_baseline(budget_s=12.0):
 
 def sweep_leg(args, local):
     """Fig. 5 analog (NEXT-2): search playouts/s vs total GPU
-    threads for leaf parallelism and block parallelism with 32- and 128-thread
-    blocks, time mode from the opening. One JSON line per point, rank 0 only."""
+    threads for leaf parallelism, block parallelism with 32- and 128-thread
+    blocks and the NEXT-4 shared tree with 128-thread workers ("trees" =
+    workers, "iterations_per_tree" = per worker), time mode from the opening.
+    One JSON line, rank 0 only."""
     import torch
     import paper_conf_ipps_rockis11_b200 as pkg
     torch.cuda.set_device(local)
     stream = torch.cuda.current_stream()
     root = pkg.position(*pkg.OPENING)
     st = torch.zeros(198, dtype=torch.int64, device="cuda")
-    handles = {"block": pkg.Mcts(scheme="block", device=local), "leaf": pkg.Mcts(scheme="leaf", device=local)}
+    handles = {"block": pkg.Mcts(scheme="block", device=local), "leaf": pkg.Mcts(scheme="leaf", device=local),
+               "tree": pkg.Mcts(scheme="tree", device=local)}
     points = []
     for total in [128, 512, 2048, 8192, 16384, 37888, 75776, 151552]:
-        for scheme, bs in [("leaf", 128), ("block", 32), ("block", 128)]:
+        for scheme, bs in [("leaf", 128), ("block", 32), ("block", 128), ("tree", 128)]:
             if scheme == "leaf" and total > 65536:
                 continue
             n_trees, threads = (1, total) if scheme == "leaf" else (total // bs, bs)
@@ -196,7 +199,8 @@ def sweep_leg(args, local):
             s = st.cpu().numpy()
             points.append({"scheme": scheme, "block": bs, "gpu_threads": total, "trees": n_trees,
                            "playouts_per_s": float(s[195]) / (ms / 1e3),
-                           "iterations_per_tree": float(s[196]) / n_trees, "ms": ms})
+                           "iterations_per_tree": float(s[196]) / n_trees, "ms": ms,
+                           "plies_per_s": float(s[197]) / (ms / 1e3)})
             if args.sweep_games and total in (512, 2048, 16384, 151552):
                 def gpu_move(black, white, to_move, seed, h=h, n_trees=n_trees, threads=threads):
                     h.search_async(pkg.position(black, white, to_move), 0, args.move_ms, n_trees, threads,
