@@ -25,6 +25,7 @@ import tempfile
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
+STATS_LEN = 199  # include/mcts.h MCTS_STATS_LEN
 sys.path.insert(0, ROOT)
 
 N_LEAVES, N_PER_LEAF, GEN_SEED, LMIN, LMAX = 4096, 256, 2, 20, 40
@@ -178,7 +179,7 @@ def sweep_leg(args, local):
     torch.cuda.set_device(local)
     stream = torch.cuda.current_stream()
     root = pkg.position(*pkg.OPENING)
-    st = torch.zeros(198, dtype=torch.int64, device="cuda")
+    st = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
     handles = {"block": pkg.Mcts(scheme="block", device=local), "leaf": pkg.Mcts(scheme="leaf", device=local),
                "tree": pkg.Mcts(scheme="tree", device=local)}
     points = []
@@ -230,6 +231,7 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
     import oracle
     res = {"W": 0, "D": 0, "L": 0}
     diffs, gpu_po, cpu_po, steps = [], [], [], []
+    depth = {"gpu": {}, "opp": {}}  # game step -> mean tree depths (searchers that report one)
     t_start = time.time()
     for g in range(games):
         gpu_color = g % 2
@@ -245,11 +247,15 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
                 continue
             seed = seed_base + 1000 * g + ply
             if to_move == gpu_color:
-                mv, po = gpu_move(black, white, to_move, seed)
+                mv, po, *dp = gpu_move(black, white, to_move, seed)
                 gpu_po.append(po)
+                if dp:
+                    depth["gpu"].setdefault(ply, []).append(dp[0])
             elif opp_move is not None:  # another device searcher (--h2h)
-                mv, po = opp_move(black, white, to_move, seed + 500)
+                mv, po, *dp = opp_move(black, white, to_move, seed + 500)
                 cpu_po.append(po)
+                if dp:
+                    depth["opp"].setdefault(ply, []).append(dp[0])
             else:
                 st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cpu_threads, move_ms, seed)
                 cpu_po.append(int(st[195]))
@@ -278,6 +284,9 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
             "point_diff_per_step": per_step,
             "gpu_playouts_per_move": float(np.mean(gpu_po)) if gpu_po else None,
             "cpu_playouts_per_move": float(np.mean(cpu_po)) if cpu_po else None,
+            # mean depth of the simulated node per game step (the paper's Fig. 8 "Depth")
+            "gpu_depth_per_step": {int(k): float(np.mean(v)) for k, v in sorted(depth["gpu"].items())},
+            "opp_depth_per_step": {int(k): float(np.mean(v)) for k, v in sorted(depth["opp"].items())},
             "wall_s": time.time() - t_start}
 
 
@@ -292,7 +301,7 @@ def h2h_leg(args, local):
     import paper_conf_ipps_rockis11_b200 as pkg
     torch.cuda.set_device(local)
     stream = torch.cuda.current_stream()
-    st = torch.zeros(198, dtype=torch.int64, device="cuda")
+    st = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
     a, b = args.h2h_schemes.split(",")
     ha = pkg.Mcts(c_uct=args.c_uct, scheme=a, device=local)
     hb = pkg.Mcts(c_uct=args.c_uct, scheme=b, device=local)
@@ -303,13 +312,15 @@ def h2h_leg(args, local):
                            st.data_ptr(), stream)
             torch.cuda.synchronize()
             x = st.cpu().numpy()
-            return pkg.best_move(x), int(x[195])
+            return pkg.best_move(x), int(x[195]), float(x[198]) / max(int(x[196]), 1)
         return move
 
     r = play_match(mover(ha, *SCHEME_SHAPE[a]), 0, args.selfplay, args.move_ms, tag="h2h",
                    opp_move=mover(hb, *SCHEME_SHAPE[b]))
     r[f"{a}_playouts_per_move"] = r.pop("gpu_playouts_per_move")
     r[f"{b}_playouts_per_move"] = r.pop("cpu_playouts_per_move")
+    r[f"{a}_depth_per_step"] = r.pop("gpu_depth_per_step")
+    r[f"{b}_depth_per_step"] = r.pop("opp_depth_per_step")
     names = {"block": "block parallelism", "leaf": "leaf parallelism", "tree": "tree parallelism"}
     shape = {k: f"{SCHEME_DESC[k]}: {v[0]} {'workers' if k == 'tree' else 'trees'} x {v[1]} threads"
              for k, v in SCHEME_SHAPE.items()}
@@ -343,7 +354,7 @@ def selfplay_leg(args, world, rank, local):
     n_trees, threads = SCHEME_SHAPE[scheme]
     m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
     stream = torch.cuda.current_stream()
-    stats = torch.zeros(198, dtype=torch.int64, device="cuda")
+    stats = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
     msg = torch.zeros(4, dtype=torch.int64, device="cuda")  # black, white, to_move, seed/-1
 
     def search(black, white, to_move, seed):
@@ -351,14 +362,14 @@ def selfplay_leg(args, world, rank, local):
         if hybrid:  # NEXT-1: GPU trees + one host tree per host core, root sums merged
             r = m.search_hybrid(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads,
                                 seed=seed, cpu_threads=len(os.sched_getaffinity(0)))
-            return r["best_move"], r["root_visits"]
+            return r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1)
         m.search_async(pos, 0, args.move_ms, n_trees, threads, seed, rank * n_trees,
                        stats.data_ptr(), stream)
         with torch.cuda.stream(stream):
             merge_root_stats(stats)
         torch.cuda.synchronize()
         st = stats.cpu().numpy()
-        return best_move_from(st), int(st[195])
+        return best_move_from(st), int(st[195]), float(st[198]) / max(int(st[196]), 1)
 
     if rank != 0:  # follower ranks: search whatever position rank 0 broadcasts
         while True:
@@ -593,7 +604,7 @@ def main():
     def run_search(handle, n_trees, threads, id_base, it_scale=1):
         # it_scale: the shared tree's iteration budget is a total over its workers
         root = pkg.position(*pkg.OPENING)
-        st = torch.zeros(198, dtype=torch.int64, device="cuda")
+        st = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
         it, ms = (args.search_iters * it_scale, 0.0) if args.search_iters else (0, args.search_ms)
         handle.search_async(root, min(it, 2) if it else 0, 0.0 if it else 20.0, n_trees, threads,
                             1000, id_base, st.data_ptr(), stream)  # warm-up: pool + ln table
@@ -620,6 +631,7 @@ def main():
             "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
+            "mean_depth": float(st[198]) / max(float(st[196]), 1.0),
             # the playout kernel's measured instructions per ply (the search
             # kernel's playouts run the same loop), per GPU
             "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ops_per_ply("playouts")[0]
@@ -632,7 +644,7 @@ def main():
             "workload": f"configs[3]: 1 tree x {LEAF_THREADS} threads per leaf batch per GPU, {mode}",
             "playouts_per_s": float(lt[195]) / (l_ms / 1e3), "ms": l_ms,
             "iterations": float(lt[196]) / world, "plies_per_s": float(lt[197]) / (l_ms / 1e3),
-            "best_move": int(pkg.best_move(lt)),
+            "best_move": int(pkg.best_move(lt)), "mean_depth": float(lt[198]) / max(float(lt[196]), 1.0),
         }
         ml.close()
         log('mt = pkg.Mcts(')
@@ -643,7 +655,7 @@ def main():
                         f"threads per GPU, {mode}, opening root, C=1.0",
             "playouts_per_s": float(tt[195]) / (t_ms / 1e3), "ms": t_ms,
             "iterations": float(tt[196]) / world, "plies_per_s": float(tt[197]) / (t_ms / 1e3),
-            "best_move": int(pkg.best_move(tt)),
+            "best_move": int(pkg.best_move(tt)), "mean_depth": float(tt[198]) / max(float(tt[196]), 1.0),
         }
         mt.close()
 

@@ -101,8 +101,11 @@ typedef struct {
  *   [130,195) root-child draws
  *   [195]     root visits (= playouts simulated)
  *   [196]     UCT iterations (summed over trees)
- *   [197]     playout plies (non-pass moves simulated)                    */
-#define MCTS_STATS_LEN 198
+ *   [197]     playout plies (non-pass moves simulated)
+ *   [198]     sum over iterations of the simulated node's depth (edges
+ *             from the root; mean tree depth = [198] / [196], the paper's
+ *             "Depth" of Fig. 8)                               */
+#define MCTS_STATS_LEN 199
 
 typedef struct {
   uint64_t visits[65];
@@ -111,6 +114,7 @@ typedef struct {
   uint64_t root_visits;
   uint64_t iterations_done;
   uint64_t plies;
+  uint64_t depth_sum; /* [198]: sum over iterations of the simulated node's depth */
   int32_t best_move; /* argmax visits, lowest index on ties (R8); -1 if the root is terminal */
   int32_t reserved;
 } mcts_root_stats;

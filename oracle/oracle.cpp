@@ -235,6 +235,7 @@ double ucb(uint64_t w, uint64_t n, double ln_parent, double C) {
 struct TreeResult {
   std::vector<Node> nodes;
   uint64_t iterations = 0;
+  uint64_t depth_sum = 0;  // sum over iterations of the simulated node's depth (edges from the root)
 };
 
 // One tree of the search: `iterations` UCT iterations with `unit` playouts per
@@ -306,6 +307,7 @@ void search_tree(uint64_t root_own, uint64_t root_opp, uint32_t unit, uint64_t i
         if (r > 0) ++wins; else if (r == 0) ++draws; else ++losses;
       }
     }
+    out->depth_sum += path.size() - 1;  // the paper's tree depth (Fig. 8)
     // 4) Backpropagation (L196-L199): the leaf's mover is the opponent of the
     // leaf's side to move, so it collects `losses`; roles alternate upwards.
     uint64_t mover_wins = losses, other_wins = wins;
@@ -422,14 +424,15 @@ double orc_ucb(uint64_t w, uint64_t n, double ln_parent, double C) { return ucb(
 
 // Full search (the mcts_search contract, iteration mode). stats layout:
 // [0,65) visits, [65,130) wins (for the root's side to move), [130,195) draws,
-// [195] root visits, [196] iterations; summed over trees tree_id_base ..
+// [195] root visits, [196] iterations, [197] playout plies, [198] sum over
+// iterations of the simulated node's depth; summed over trees tree_id_base ..
 // tree_id_base + n_trees - 1. capacity = max nodes per tree (0 = iterations+1).
 // Returns best move (max visits, lowest index on ties) or -1 if the root is
 // terminal. plies_out (nullable) receives the playout plies.
 int orc_uct_search(const orc_position* root, uint32_t n_trees, uint32_t unit, uint64_t iterations,
                    uint64_t seed, uint32_t tree_id_base, double C, uint64_t capacity,
                    int64_t* stats, uint64_t* plies_out, int nthreads) {
-  for (int i = 0; i < 197; ++i) stats[i] = 0;
+  for (int i = 0; i < 199; ++i) stats[i] = 0;
   uint64_t own, opp;
   to_own_opp(*root, &own, &opp);
   if (capacity == 0) capacity = iterations + 1;
@@ -462,8 +465,10 @@ int orc_uct_search(const orc_position* root, uint32_t n_trees, uint32_t unit, ui
     }
     stats[195] += (int64_t)nodes[0].n;
     stats[196] += (int64_t)res[t].iterations;
+    stats[198] += (int64_t)res[t].depth_sum;
     ptot += plies[t];
   }
+  stats[197] = (int64_t)ptot;
   if (plies_out) *plies_out = ptot;
   if (res.empty() || res[0].nodes[0].terminal) return -1;
   int best = -1;
@@ -547,7 +552,7 @@ void orc_gen_positions(uint64_t seed, uint32_t n, uint32_t lmin, uint32_t lmax, 
 // stats as in orc_uct_search. Returns the chosen move (-1 terminal).
 int orc_mcts_timed(const orc_position* root, int nthreads, double budget_ms, uint64_t seed,
                    double C, int64_t* stats) {
-  for (int i = 0; i < 197; ++i) stats[i] = 0;
+  for (int i = 0; i < 199; ++i) stats[i] = 0;
   uint64_t own, opp;
   to_own_opp(*root, &own, &opp);
   Node r0 = make_node(own, opp, -1, -1);

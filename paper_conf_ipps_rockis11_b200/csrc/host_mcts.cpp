@@ -3,6 +3,7 @@
 // (R1-R10) with one simulation per iteration; used only by
 // mcts_search_hybrid, never as a substitute for the GPU.
 #include "host_mcts.h"
+#include "../../include/mcts.h"
 
 #include <atomic>
 #include <chrono>
@@ -121,7 +122,7 @@ void run_tree(const HostSearchArgs& a, u32 t, int64_t* st) {
   Tree T;
   T.add(a.own, a.opp, 0xFFu);
   if (T.term[0]) return;
-  u64 plies = 0;
+  u64 plies = 0, depth_sum = 0;
   u64 it = 0;
   std::vector<u32> path;
   for (; it < a.iterations; ++it) {
@@ -167,6 +168,7 @@ void run_tree(const HostSearchArgs& a, u32 t, int64_t* st) {
       v = c;
       path.push_back(v);
     }
+    depth_sum += path.size() - 1;
     int r;  // simulation (one per iteration)
     if (T.term[v]) {
       const int x = popc(T.own[v]), y = popc(T.opp[v]);
@@ -192,14 +194,15 @@ void run_tree(const HostSearchArgs& a, u32 t, int64_t* st) {
   st[195] += T.k[0];
   st[196] += (int64_t)it;
   st[197] += (int64_t)plies;
+  st[198] += (int64_t)depth_sum;
 }
 
 }  // namespace
 
 void search(const HostSearchArgs& a, int64_t* stats) {
-  for (int i = 0; i < 198; ++i) stats[i] = 0;
+  for (int i = 0; i < MCTS_STATS_LEN; ++i) stats[i] = 0;
   const u32 T = a.threads ? a.threads : 1;
-  std::vector<std::vector<int64_t>> part(T, std::vector<int64_t>(198, 0));
+  std::vector<std::vector<int64_t>> part(T, std::vector<int64_t>(MCTS_STATS_LEN, 0));
   std::atomic<u32> next{0};
   auto worker = [&](u32 tid) {
     for (;;) {
@@ -213,7 +216,7 @@ void search(const HostSearchArgs& a, int64_t* stats) {
   worker(0);
   for (auto& th : pool) th.join();
   for (u32 i = 0; i < T; ++i)
-    for (int j = 0; j < 198; ++j) stats[j] += part[i][j];
+    for (int j = 0; j < MCTS_STATS_LEN; ++j) stats[j] += part[i][j];
 }
 
 }  // namespace mcts_host

@@ -154,6 +154,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
 
   u32 plies = 0;
   u32 it = 0;
+  unsigned long long depth_sum = 0;  // lane 0 of warp 0: sum of leaf depths (Fig. 8 "Depth")
   if (!meta_term(T.meta[base])) {
     for (;; ++it) {
       if (warp == 0) {
@@ -167,6 +168,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
           const LeafInfo L = select_expand(T, base, path, &s_slot_used, a.lnT, unit, a.C, lane);
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth;
+            depth_sum += (unsigned)L.depth;
           }
         }
         if (lane == 0) s_stop = stop;
@@ -201,6 +203,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
     unsigned long long P = lane < nwarps ? s_w[lane] : 0u;
     for (int off = 16; off > 0; off >>= 1) P += __shfl_xor_sync(kFull, P, off);
     if (lane == 0 && P) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, P);
+    if (lane == 0 && depth_sum) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
     merge_root(T, base, unit, it, a.stats, lane);
   }
 }
@@ -243,6 +246,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   __syncthreads();
   u32 plies = 0;
   u32 it = 0;
+  unsigned long long depth_sum = 0;  // leader lane 0
   for (;; ++it) {
     if (leader) {
       if (it > 0) {
@@ -260,7 +264,10 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       stop = __shfl_sync(kFull, stop, 0);
       if (!stop) {
         const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
-        if (lane == 0) { s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term; }
+        if (lane == 0) {
+          s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
+          depth_sum += (unsigned)L.depth;
+        }
       }
       if (lane == 0) S->stop = stop;
     }
@@ -289,6 +296,8 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   }
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
+  if (leader && lane == 0 && depth_sum)
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
 

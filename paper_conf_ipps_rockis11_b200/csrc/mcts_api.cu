@@ -537,6 +537,7 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   out->root_visits = (uint64_t)hs[195];
   out->iterations_done = (uint64_t)hs[196];
   out->plies = (uint64_t)hs[197];
+  out->depth_sum = (uint64_t)hs[198];
   out->best_move = mcts_best_move((const int64_t*)hs);
   out->reserved = 0;
   return MCTS_OK;
@@ -551,6 +552,7 @@ static void fill_root_stats(const long long* hs, mcts_root_stats* out) {
   out->root_visits = (uint64_t)hs[195];
   out->iterations_done = (uint64_t)hs[196];
   out->plies = (uint64_t)hs[197];
+  out->depth_sum = (uint64_t)hs[198];
   out->best_move = mcts_best_move((const int64_t*)hs);
   out->reserved = 0;
 }

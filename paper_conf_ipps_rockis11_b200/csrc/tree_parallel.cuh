@@ -25,7 +25,7 @@
 //   * backpropagation: atomic adds of (k, w, d) along the path, then vl -= 1.
 // With W = 1 nothing races, the virtual-loss terms are zero at every read and
 // the search is the sequential UCT of the oracle with one tree, bit for bit
-// (tests/test_gpu_parity.py). With W > 1 the result depends on timing (as on
+// (tests/test_gpu_tree.py). With W > 1 the result depends on timing (as on
 // any parallel machine): tests check the tree invariants (tree_check_kernel).
 //
 // All tree fields are read with L1-bypassing loads (ld.relaxed/acquire.gpu):
@@ -235,6 +235,7 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
 
   u32 plies = 0;
   u32 done = 0;
+  unsigned long long depth_sum = 0;  // lane 0 of warp 0
   if (!meta_term(ld_acq(&T.meta[0]))) {
     for (;;) {
       if (warp == 0) {
@@ -252,6 +253,7 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
           const LeafInfo L = tree_select_expand(T, S, path, a.lnT, unit, a.C, lane);
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth; s_it = it;
+            depth_sum += (unsigned)L.depth;
           }
         }
         if (lane == 0) s_stop = stop;
@@ -288,6 +290,7 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
     unsigned long long* st = reinterpret_cast<unsigned long long*>(a.stats);
     if (lane == 0 && P) atomicAdd(st + 197, P);
     if (lane == 0 && done) atomicAdd(st + 196, (unsigned long long)done);
+    if (lane == 0 && depth_sum) atomicAdd(st + 198, depth_sum);
   }
 }
 

@@ -12,6 +12,8 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
+from ._native import STATS_LEN
+
 
 def tree_id_base(rank: int, n_trees_per_rank: int) -> int:
     return rank * n_trees_per_rank
@@ -44,7 +46,7 @@ def search(mcts, root, n_trees: int, threads_per_tree: int, seed: int, iteration
            time_ms: float = 0.0, group=None, stream=None) -> dict:
     """Block-parallel search on this rank's GPU + the root-stats allreduce."""
     rank = dist.get_rank(group) if dist.is_available() and dist.is_initialized() else 0
-    stats = torch.zeros(198, dtype=torch.int64, device=f"cuda:{mcts.device}")
+    stats = torch.zeros(STATS_LEN, dtype=torch.int64, device=f"cuda:{mcts.device}")
     s = stream if stream is not None else torch.cuda.current_stream()
     mcts.search_async(root, iterations, time_ms, n_trees, threads_per_tree, seed,
                       tree_id_base(rank, n_trees), stats.data_ptr(), s)

@@ -44,7 +44,7 @@ def test_sass_is_sm100a():
 def test_best_move_host_helper():
     import numpy as np
     import paper_conf_ipps_rockis11_b200 as pkg
-    s = np.zeros(198, dtype=np.int64)
+    s = np.zeros(pkg.STATS_LEN, dtype=np.int64)
     assert pkg.best_move(s) == -1
     s[[19, 26, 37]] = [5, 9, 9]
     assert pkg.best_move(s) == 26

@@ -12,6 +12,8 @@ import torch
 import paper_conf_ipps_rockis11_b200 as pkg
 from paper_conf_ipps_rockis11_b200 import device as dev
 
+STATS_LEN = pkg.STATS_LEN
+
 pytestmark = pytest.mark.gpu
 
 
@@ -141,7 +143,7 @@ def test_playouts_leaf_range_sharding(mcts, orc):
 
 # ---------------------------------------------------------------- search
 def _cmp_search(res, ostats, obest):
-    assert res["stats"][:197].tolist() == ostats[:197].tolist()
+    assert res["stats"][:199].tolist() == ostats[:199].tolist()
     assert res["best_move"] == obest
 
 
@@ -184,8 +186,8 @@ def test_search_async_tree_id_base_merge_identity(mcts, orc):
     root = orc.gen_positions(13, 1, 20, 40)
     n, k = 37, 4
     whole = mcts.search(root, iterations=15, n_trees=n * k, threads_per_tree=64, seed=9)
-    acc = torch.zeros(198, dtype=torch.int64, device="cuda")
-    part = torch.zeros(198, dtype=torch.int64, device="cuda")
+    acc = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
+    part = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
     for r in range(k):
         mcts.search_async(root, 15, 0.0, n, 64, 9, r * n, part.data_ptr(), torch.cuda.current_stream())
         acc += part
@@ -194,7 +196,7 @@ def test_search_async_tree_id_base_merge_identity(mcts, orc):
     ostats, _, _ = orc.uct_search(root, n, 64, 15, 9, tree_id_base=2 * n)
     mcts.search_async(root, 15, 0.0, n, 64, 9, 2 * n, part.data_ptr(), torch.cuda.current_stream())
     torch.cuda.synchronize()
-    assert part.cpu().numpy()[:197].tolist() == ostats[:197].tolist()
+    assert part.cpu().numpy()[:199].tolist() == ostats[:199].tolist()
 
 
 def test_search_leaf_bit_exact(mcts_leaf, orc):
@@ -333,10 +335,10 @@ def test_search_hybrid_iteration_mode(mcts, orc):
     res = mcts.search_hybrid(root, iterations=40, n_trees=6, threads_per_tree=64, seed=12, cpu_threads=3)
     g, _, gp = orc.uct_search(root, 6, 64, 40, 12)
     c, _, cp = orc.uct_search(root, 3, 1, 40, 12, tree_id_base=0x40000000)
-    assert res["cpu"]["stats"][:197].tolist() == c[:197].tolist()
+    assert res["cpu"]["stats"][:199].tolist() == c[:199].tolist()
     assert res["cpu"]["plies"] == cp
     merged = g + c
-    assert res["stats"][:197].tolist() == merged[:197].tolist()
+    assert res["stats"][:199].tolist() == merged[:199].tolist()
     assert res["best_move"] == int(np.argmax(merged[:65]))
     assert res["plies"] == gp + cp
 

@@ -153,3 +153,26 @@ def test_pass_root(orc):
     black, white = 0b11, 0b100
     s, best, _ = orc.uct_search(orc.position(black, white, 1), 2, 32, 3, seed=1)
     assert best == 64 and s[64] == 2 * 3 * 32 and s[:64].sum() == 0
+
+
+def test_depth_sum_hand_trace(orc):
+    """stats[198] = sum over iterations of the simulated node's depth (the
+    paper's tree depth, Fig. 8). From the opening the first four iterations
+    expand the four root children (depth 1 each) and the fifth expands a child
+    of the selected one (depth 2): 1 + 1 + 1 + 1 + 2 = 6."""
+    s4, _, _ = orc.uct_search(orc.opening(), 1, 64, 4, seed=1)
+    s5, _, p5 = orc.uct_search(orc.opening(), 1, 64, 5, seed=1)
+    assert s4[198] == 4 and s5[198] == 6
+    assert s5[197] == p5  # [197] = playout plies, also returned separately
+
+
+@pytest.mark.parametrize("seed,unit,iters,cap", [(1, 32, 300, 0), (2, 1, 2000, 0), (5, 32, 200, 40)])
+def test_depth_sum_equals_tree_visits(orc, seed, unit, iters, cap):
+    """Every iteration adds `unit` to n of each node on its path below the root,
+    so the depth sum equals sum over non-root nodes of n / unit (the tree dump
+    against the search's own depth bookkeeping, incl. a full pool)."""
+    for p in orc.gen_positions(seed, 2, 10, 40):
+        root = np.array([p])
+        s, _, _ = orc.uct_search(root, 1, unit, iters, seed, tree_id_base=seed, capacity=cap)
+        t = orc.uct_tree(root, unit, iters, seed, tree_id=seed, C=1.0, capacity=cap)
+        assert int(s[198]) == sum(int(x) for x in t["n"][1:]) // unit
