@@ -24,7 +24,9 @@
 // Random123 Philox known-answer vectors, closed-form pick-bucket counts, the
 // exact random-play outcome distribution of small endgames, a 45-digit decimal
 // ln reference, high-precision UCB values, a hand trace of the first UCT
-// iterations, tree invariants and the multi-tree merge identity.
+// iterations (incl. the depth sum of the paper's Fig. 8 "Depth", L490-L511),
+// tree invariants, depth sum = sum of non-root visits / unit, and the
+// multi-tree merge identity.
 //
 // Deliberately NOT tuned: move generation walks every empty square in every
 // direction with (row, col) coordinates; every RNG word recomputes Philox.
