@@ -74,3 +74,28 @@ def test_play_match_two_device_players_bookkeeping():
     assert r["mean_disc_diff"] == sum(want) / 2
     assert r["results"]["W"] == sum(d > 0 for d in want)
     assert r["point_diff_per_step"][-1] == sum(want) / 2
+
+
+def test_play_match_depth_per_step():
+    """Searchers may return (move, playouts, mean depth); play_match averages the
+    depth per game step (ply index) over games, separately for each side
+    (Fig. 8 analog). Here side A reports depth = ply index, side B none."""
+    import oracle
+    seen = []
+
+    def a(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        m = oracle.legal(own, opp)
+        ply = bin(black | white).count("1") - 4  # every move adds one disc
+        seen.append(ply)
+        return (m & -m).bit_length() - 1, 1, float(ply)
+
+    def b(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        return oracle.legal(own, opp).bit_length() - 1, 1
+
+    r = bench.play_match(a, 0, 2, 1.0, opp_move=b)
+    dp = r["gpu_depth_per_step"]
+    assert dp and all(v == float(k) for k, v in dp.items())
+    assert sorted(dp) == sorted(set(seen))
+    assert r["opp_depth_per_step"] == {}
