@@ -44,7 +44,9 @@ def best_move_from(stats) -> int:
 
 def search(mcts, root, n_trees: int, threads_per_tree: int, seed: int, iterations: int = 0,
            time_ms: float = 0.0, group=None, stream=None) -> dict:
-    """Block-parallel search on this rank's GPU + the root-stats allreduce."""
+    """This rank's search (the handle's scheme) + the root-stats allreduce. For
+    MCTS_TREE each rank grows one shared tree with Philox c0 = rank * n_trees
+    (root parallelism across GPUs, tree parallelism inside one)."""
     rank = dist.get_rank(group) if dist.is_available() and dist.is_initialized() else 0
     stats = torch.zeros(STATS_LEN, dtype=torch.int64, device=f"cuda:{mcts.device}")
     s = stream if stream is not None else torch.cuda.current_stream()
