@@ -221,7 +221,7 @@ def sweep_leg(args, local):
                       "points": points}), flush=True)
 
 
-def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", opp_move=None):
+def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", opp_move=None, cpu_c=1.0):
     """Games of the B200 searcher (gpu_move(black, white, to_move, seed) ->
     (move, playouts)) against the oracle's root-parallel CPU MCTS on
     `cpu_threads` host threads, alternating colours, equal time per move; the
@@ -257,7 +257,8 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
                 if dp:
                     depth["opp"].setdefault(ply, []).append(dp[0])
             else:
-                st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cpu_threads, move_ms, seed)
+                st, mv = oracle.mcts_timed(oracle.position(black, white, to_move), cpu_threads, move_ms, seed,
+                                           C=cpu_c)
                 cpu_po.append(int(st[195]))
             assert 0 <= mv < 64 and (legal >> mv) & 1, (mv, hex(legal))
             f = oracle.flips(own, opp, mv)
@@ -391,25 +392,26 @@ def selfplay_leg(args, world, rank, local):
         return search(black, white, to_move, seed)
 
     cores = len(os.sched_getaffinity(0))
+    cpu_c = args.c_uct if args.cpu_c is None else args.cpu_c
     workload = (f"{SCHEME_DESC[scheme]} searcher ({n_trees} {'workers' if scheme == 'tree' else 'trees'} x "
                 f"{threads} threads per GPU, {args.sp_scheme}, {world} GPU(s))")
     if args.fig7:
         curves = []
         t = 1
         while t <= cores:
-            r = play_match(gpu_move, t, args.selfplay, args.move_ms, tag=f"cpu{t}")
+            r = play_match(gpu_move, t, args.selfplay, args.move_ms, tag=f"cpu{t}", cpu_c=cpu_c)
             curves.append({"cpu_threads": t, **r})
             t *= 2
         out = {"metric": "point difference per game step vs root-parallel CPU MCTS on 1..N host threads "
                          "(Fig. 7 analog)", "unit": "discs", "n_gpus": world,
                "config": {"workload": workload, "move_ms": args.move_ms, "games_per_point": args.selfplay,
-                          "C": args.c_uct}, "curves": curves}
+                          "C": args.c_uct, "C_cpu": cpu_c}, "curves": curves}
     else:
-        r = play_match(gpu_move, cores, args.selfplay, args.move_ms)
+        r = play_match(gpu_move, cores, args.selfplay, args.move_ms, cpu_c=cpu_c)
         out = {"metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": r["win_pct"],
                "unit": "%", "n_gpus": world,
                "config": {"workload": workload + f" vs root-parallel CPU oracle MCTS on {cores} host threads",
-                          "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct}, **r}
+                          "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct, "C_cpu": cpu_c}, **r}
     if world > 1:
         msg.copy_(torch.tensor([0, 0, 0, -1]))
         dist.broadcast(msg, 0)
@@ -451,6 +453,8 @@ def main():
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
+    ap.add_argument("--cpu-c", type=float, default=None,
+                    help="UCB constant of the CPU oracle opponent (default: the same as --c-uct)")
     ap.add_argument("--h2h", action="store_true",
                     help="with --selfplay: head-to-head of two device searchers on one GPU (--h2h-schemes)")
     ap.add_argument("--h2h-schemes", default="block,leaf",
