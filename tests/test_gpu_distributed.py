@@ -20,7 +20,7 @@ def _free_port():
     return p
 
 
-def _rank(rank, world, port, q):
+def _rank(rank, world, port, q, scheme, n_trees):
     import torch
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -30,29 +30,32 @@ def _rank(rank, world, port, q):
         import paper_conf_ipps_rockis11_b200 as pkg
         from paper_conf_ipps_rockis11_b200 import distributed
         torch.cuda.set_device(0)
-        m = pkg.Mcts(c_uct=1.0, scheme="block", device=0)
+        m = pkg.Mcts(c_uct=1.0, scheme=scheme, device=0)
         root = np.zeros(1, dtype=pkg.POSITION_DTYPE)
         root["black"], root["white"], root["to_move"] = 0x0000000810000000, 0x0000001008000000, 0
-        r = distributed.search(m, root, n_trees=24, threads_per_tree=64, seed=11, iterations=12)
+        r = distributed.search(m, root, n_trees=n_trees, threads_per_tree=64, seed=11, iterations=12)
         q.put((rank, r["stats"].tolist(), r["best_move"]))
         m.close()
     finally:
         dist.destroy_process_group()
 
 
-def test_two_rank_allreduce_matches_single_search(orc):
+@pytest.mark.parametrize("scheme,n_trees", [("block", 24), ("tree", 1)])
+def test_two_rank_allreduce_matches_single_search(orc, scheme, n_trees):
+    """block: 24 trees per rank; tree: one one-worker shared tree per rank
+    (c0 = rank), i.e. root parallelism across ranks over tree-parallel GPUs."""
     world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_rank, args=(r, world, port, q)) for r in range(world)]
+    ps = [ctx.Process(target=_rank, args=(r, world, port, q, scheme, n_trees)) for r in range(world)]
     for p in ps:
         p.start()
     res = [q.get(timeout=600) for _ in range(world)]
     for p in ps:
         p.join(timeout=120)
         assert p.exitcode == 0
-    ostats, obest, _ = orc.uct_search(orc.opening(), 24 * world, 64, 12, 11)
+    ostats, obest, _ = orc.uct_search(orc.opening(), n_trees * world, 64, 12, 11)
     for rank, stats, best in res:
         assert stats[:199] == ostats[:199].tolist()
         assert best == obest
