@@ -9,8 +9,9 @@ playouts, inputs resident in HBM, launched through mcts_playouts_async. N>1:
 one process per GPU (torchrun), every rank runs its own batch with distinct
 playout streams (leaf_id_base = rank * 4096): weak scaling, no collective on
 the data path. The block-parallel search (configs[2] shape, a1-a11 incl. the
-NCCL root-stats allreduce at N>1) and the leaf-parallel comparison (configs[3])
-are reported in the "search" / "leaf_search" objects of the same line.
+NCCL root-stats allreduce at N>1), the leaf-parallel comparison (configs[3])
+and the NEXT-4 shared tree (1184 workers x 128 threads on one tree) are reported
+in the "search" / "leaf_search" / "tree_search" objects of the same line.
 
 Prints ONE JSON line on rank 0. See DESIGN.md §8 for every field.
 """
