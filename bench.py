@@ -408,11 +408,12 @@ def selfplay_leg(args, world, rank, local):
                "config": {"workload": workload, "move_ms": args.move_ms, "games_per_point": args.selfplay,
                           "C": args.c_uct, "C_cpu": cpu_c}, "curves": curves}
     else:
-        r = play_match(gpu_move, cores, args.selfplay, args.move_ms, cpu_c=cpu_c)
+        r = play_match(gpu_move, cores, args.selfplay, args.move_ms, seed_base=args.sp_seed_base, cpu_c=cpu_c)
         out = {"metric": "win% vs CPU-oracle MCTS (equal wall time per move)", "value": r["win_pct"],
                "unit": "%", "n_gpus": world,
                "config": {"workload": workload + f" vs root-parallel CPU oracle MCTS on {cores} host threads",
-                          "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct, "C_cpu": cpu_c}, **r}
+                          "move_ms": args.move_ms, "colours": "alternating", "C": args.c_uct, "C_cpu": cpu_c,
+                          "seed_base": args.sp_seed_base}, **r}
     if world > 1:
         msg.copy_(torch.tensor([0, 0, 0, -1]))
         dist.broadcast(msg, 0)
@@ -454,6 +455,9 @@ def main():
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
+    ap.add_argument("--sp-seed-base", type=int, default=1000,
+                    help="self-play seed base (game g, ply p uses seed_base + 1000 g + p): a new base gives "
+                         "an independent game set to pool with earlier ones")
     ap.add_argument("--cpu-c", type=float, default=None,
                     help="UCB constant of the CPU oracle opponent (default: the same as --c-uct)")
     ap.add_argument("--h2h", action="store_true",

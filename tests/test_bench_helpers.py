@@ -99,3 +99,29 @@ def test_play_match_depth_per_step():
     assert dp and all(v == float(k) for k, v in dp.items())
     assert sorted(dp) == sorted(set(seen))
     assert r["opp_depth_per_step"] == {}
+
+
+def test_play_match_seed_base():
+    """--sp-seed-base: game g, ply p hands seed_base + 1000 g + p to the
+    searcher (the opponent gets +500), so two bases give disjoint seed sets."""
+    import oracle
+    got = {}
+
+    def mover(tag):
+        def f(black, white, to_move, seed):
+            got.setdefault(tag, []).append(seed)
+            own, opp = (black, white) if to_move == 0 else (white, black)
+            m = oracle.legal(own, opp)
+            return (m & -m).bit_length() - 1, 1
+        return f
+
+    bench.play_match(mover("a"), 0, 2, 1.0, seed_base=100000, opp_move=mover("b"))
+    assert min(got["a"]) >= 100000 and max(got["a"]) < 100000 + 2000
+    # the opponent's seeds are its plies' bases + 500 (plies alternate sides)
+    assert all(100000 <= s - 500 < 100000 + 2000 and (s - 500) % 1000 < 100 for s in got["b"])
+    assert set(s - 500 for s in got["b"]).isdisjoint(got["a"])
+    seeds_a = sorted(got["a"])
+    assert len(set(seeds_a)) == len(seeds_a)
+    got.clear()
+    bench.play_match(mover("a"), 0, 2, 1.0, opp_move=mover("b"))
+    assert max(got["a"]) < 100000
