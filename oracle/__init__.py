@@ -66,7 +66,7 @@ def lib() -> ctypes.CDLL:
         L.orc_uct_tree.argtypes = [vp, u32, u64, u64, u32, dbl, u64, vp, vp, vp, vp, vp, vp]
         L.orc_uct_tree.restype = ctypes.c_int64
         L.orc_gen_positions.argtypes = [u64, u32, u32, u32, vp]; L.orc_gen_positions.restype = None
-        L.orc_mcts_timed.argtypes = [vp, i32, dbl, u64, dbl, vp]; L.orc_mcts_timed.restype = i32
+        L.orc_mcts_timed.argtypes = [vp, i32, dbl, u64, dbl, vp, u64]; L.orc_mcts_timed.restype = i32
         _lib = L
     return _lib
 
@@ -180,8 +180,12 @@ def gen_positions(seed: int, n: int, lmin: int, lmax: int) -> np.ndarray:
     return out
 
 
-def mcts_timed(root: np.ndarray, nthreads: int, budget_ms: float, seed: int, C: float = 1.0):
-    """Root-parallel CPU MCTS opponent, one tree per thread."""
+def mcts_timed(root: np.ndarray, nthreads: int, budget_ms: float, seed: int, C: float = 1.0,
+               max_iterations: int = 0):
+    """Root-parallel CPU MCTS opponent, one tree per thread,
+    unit 1, grown by the same UCT iteration as uct_search. Stops at budget_ms
+    (> 0) and/or max_iterations per tree (> 0); with only the cap it equals
+    uct_search(root, nthreads, 1, max_iterations, seed) bit for bit."""
     stats = np.zeros(N_STATS, dtype=np.int64)
-    best = lib().orc_mcts_timed(_ptr(root), nthreads, budget_ms, seed, C, _ptr(stats))
+    best = lib().orc_mcts_timed(_ptr(root), nthreads, budget_ms, seed, C, _ptr(stats), max_iterations)
     return stats, int(best)

@@ -25,8 +25,10 @@
 // exact random-play outcome distribution of small endgames, a 45-digit decimal
 // ln reference, high-precision UCB values, a hand trace of the first UCT
 // iterations (incl. the depth sum of the paper's Fig. 8 "Depth", L490-L511),
-// tree invariants, depth sum = sum of non-root visits / unit, and the
-// multi-tree merge identity.
+// tree invariants, depth sum = sum of non-root visits / unit, the
+// multi-tree merge identity, the UCB operation order (R1) against five
+// re-orderings, and the CPU opponent (orc_mcts_timed, iteration-capped) equal
+// to the iteration-mode search bit for bit.
 //
 // Deliberately NOT tuned: move generation walks every empty square in every
 // direction with (row, col) coordinates; every RNG word recomputes Philox.
@@ -240,88 +242,99 @@ struct TreeResult {
   uint64_t depth_sum = 0;  // sum over iterations of the simulated node's depth (edges from the root)
 };
 
-// One tree of the search: `iterations` UCT iterations with `unit` playouts per
-// iteration, playout streams keyed (c0 = tree_id, c1 = iteration, c2 = thread).
+// One UCT iteration (number `it`) on a tree whose root is nodes[0], with `unit`
+// playouts per iteration, playout streams keyed (c0 = tree_id, c1 = it,
+// c2 = thread), ln table lnT[k] = RN(ln(k * unit)) indexed by k = parent n / unit.
+// Both the iteration-mode search (search_tree) and the CPU opponent
+// (orc_mcts_timed) grow their trees with this one function.
+void uct_iteration(TreeResult* out, uint64_t it, uint32_t unit, uint64_t seed, uint32_t tree_id,
+                   double C, uint64_t capacity, const std::vector<double>& lnT, uint64_t* plies) {
+  std::vector<Node>& nodes = out->nodes;
+  // 1) Selection (L157-L178): descend through fully expanded nodes.
+  std::vector<int> path;
+  int v = 0;
+  path.push_back(v);
+  while (!nodes[v].terminal && fully_expanded(nodes[v])) {
+    const Node& p = nodes[v];
+    double ln_parent = lnT[p.n / unit];
+    int best = -1;
+    double best_u = -INFINITY;
+    for (int c : p.children) {
+      double u = ucb(nodes[c].w, nodes[c].n, ln_parent, C);
+      if (u > best_u) { best_u = u; best = c; }
+    }
+    v = best;
+    path.push_back(v);
+  }
+  // 2) Expansion (L179-L182): one node per iteration, lowest untried move.
+  if (!nodes[v].terminal && nodes.size() < capacity) {
+    const Node& p = nodes[v];
+    int mv;
+    uint64_t cown, copp;
+    if (p.legal_moves == 0) {
+      mv = 64;  // pass child
+      cown = p.opp; copp = p.own;
+    } else {
+      int idx = (int)p.children.size(), seen = 0;
+      mv = -1;
+      for (int s = 0; s < 64; ++s) {
+        if ((p.legal_moves >> s) & 1) {
+          if (seen == idx) { mv = s; break; }
+          ++seen;
+        }
+      }
+      uint64_t f = flips(p.own, p.opp, mv);
+      uint64_t mover = p.own | f | (1ULL << mv);
+      uint64_t other = p.opp & ~f;
+      cown = other; copp = mover;
+    }
+    nodes.push_back(make_node(cown, copp, mv, v));
+    int c = (int)nodes.size() - 1;
+    nodes[v].children.push_back(c);
+    v = c;
+    path.push_back(v);
+  }
+  // 3) Simulation (L183-L195): `unit` playouts from the leaf.
+  uint64_t wins = 0, draws = 0, losses = 0;  // for the leaf's side to move
+  const Node& leaf = nodes[v];
+  if (leaf.terminal) {
+    int a = popcount64(leaf.own), b = popcount64(leaf.opp);
+    if (a > b) wins = unit; else if (a == b) draws = unit; else losses = unit;
+  } else {
+    for (uint32_t t = 0; t < unit; ++t) {
+      uint32_t pl = 0;
+      int r = playout(leaf.own, leaf.opp, seed, tree_id, (uint32_t)it, t, &pl);
+      *plies += pl;
+      if (r > 0) ++wins; else if (r == 0) ++draws; else ++losses;
+    }
+  }
+  out->depth_sum += path.size() - 1;  // the paper's tree depth (Fig. 8)
+  // 4) Backpropagation (L196-L199): the leaf's mover is the opponent of the
+  // leaf's side to move, so it collects `losses`; roles alternate upwards.
+  uint64_t mover_wins = losses, other_wins = wins;
+  for (int i = (int)path.size() - 1; i >= 0; --i) {
+    Node& x = nodes[path[i]];
+    x.n += unit;
+    x.w += mover_wins;
+    x.d += draws;
+    std::swap(mover_wins, other_wins);
+  }
+  out->iterations = it + 1;
+}
+
+// One tree of the search: `iterations` UCT iterations (uct_iteration) from a
+// fresh root.
 void search_tree(uint64_t root_own, uint64_t root_opp, uint32_t unit, uint64_t iterations,
                  uint64_t seed, uint32_t tree_id, double C, uint64_t capacity,
                  const std::vector<double>& lnT, TreeResult* out, uint64_t* plies_total) {
   std::vector<Node>& nodes = out->nodes;
   nodes.clear();
   nodes.push_back(make_node(root_own, root_opp, -1, -1));
-  if (nodes[0].terminal) { out->iterations = 0; return; }
+  out->iterations = 0;
+  if (nodes[0].terminal) return;
   uint64_t plies = 0;
-  for (uint64_t it = 0; it < iterations; ++it) {
-    // 1) Selection (L157-L178): descend through fully expanded nodes.
-    std::vector<int> path;
-    int v = 0;
-    path.push_back(v);
-    while (!nodes[v].terminal && fully_expanded(nodes[v])) {
-      const Node& p = nodes[v];
-      double ln_parent = lnT[p.n / unit];
-      int best = -1;
-      double best_u = -INFINITY;
-      for (int c : p.children) {
-        double u = ucb(nodes[c].w, nodes[c].n, ln_parent, C);
-        if (u > best_u) { best_u = u; best = c; }
-      }
-      v = best;
-      path.push_back(v);
-    }
-    // 2) Expansion (L179-L182): one node per iteration, lowest untried move.
-    if (!nodes[v].terminal && nodes.size() < capacity) {
-      const Node& p = nodes[v];
-      int mv;
-      uint64_t cown, copp;
-      if (p.legal_moves == 0) {
-        mv = 64;  // pass child
-        cown = p.opp; copp = p.own;
-      } else {
-        int idx = (int)p.children.size(), seen = 0;
-        mv = -1;
-        for (int s = 0; s < 64; ++s) {
-          if ((p.legal_moves >> s) & 1) {
-            if (seen == idx) { mv = s; break; }
-            ++seen;
-          }
-        }
-        uint64_t f = flips(p.own, p.opp, mv);
-        uint64_t mover = p.own | f | (1ULL << mv);
-        uint64_t other = p.opp & ~f;
-        cown = other; copp = mover;
-      }
-      nodes.push_back(make_node(cown, copp, mv, v));
-      int c = (int)nodes.size() - 1;
-      nodes[v].children.push_back(c);
-      v = c;
-      path.push_back(v);
-    }
-    // 3) Simulation (L183-L195): `unit` playouts from the leaf.
-    uint64_t wins = 0, draws = 0, losses = 0;  // for the leaf's side to move
-    const Node& leaf = nodes[v];
-    if (leaf.terminal) {
-      int a = popcount64(leaf.own), b = popcount64(leaf.opp);
-      if (a > b) wins = unit; else if (a == b) draws = unit; else losses = unit;
-    } else {
-      for (uint32_t t = 0; t < unit; ++t) {
-        uint32_t pl = 0;
-        int r = playout(leaf.own, leaf.opp, seed, tree_id, (uint32_t)it, t, &pl);
-        plies += pl;
-        if (r > 0) ++wins; else if (r == 0) ++draws; else ++losses;
-      }
-    }
-    out->depth_sum += path.size() - 1;  // the paper's tree depth (Fig. 8)
-    // 4) Backpropagation (L196-L199): the leaf's mover is the opponent of the
-    // leaf's side to move, so it collects `losses`; roles alternate upwards.
-    uint64_t mover_wins = losses, other_wins = wins;
-    for (int i = (int)path.size() - 1; i >= 0; --i) {
-      Node& x = nodes[path[i]];
-      x.n += unit;
-      x.w += mover_wins;
-      x.d += draws;
-      std::swap(mover_wins, other_wins);
-    }
-  }
-  out->iterations = iterations;
+  for (uint64_t it = 0; it < iterations; ++it)
+    uct_iteration(out, it, unit, seed, tree_id, C, capacity, lnT, &plies);
   if (plies_total) *plies_total += plies;
 }
 
@@ -549,89 +562,46 @@ void orc_gen_positions(uint64_t seed, uint32_t n, uint32_t lmin, uint32_t lmax, 
 }
 
 // Root-parallel CPU MCTS opponent: one tree
-// per thread, one playout per iteration (unit = 1), until the wall-clock
-// budget expires; roots summed. Not bit-reproducible (time-based).
-// stats as in orc_uct_search. Returns the chosen move (-1 terminal).
+// per thread, one playout per iteration (unit = 1), grown with the same
+// uct_iteration as the iteration-mode search; roots summed (L199-L202).
+// Thread t is tree t: streams (c0 = t, c1 = iteration, c2 = 0), exactly
+// uct_search(root, nthreads, unit 1, ..., tree_id_base 0) for the same
+// iteration counts. Stops at the wall-clock budget (budget_ms > 0; not
+// reproducible) and/or after max_iterations per tree (> 0; then with no
+// deadline it is bit-exact to uct_search(root, nthreads, 1, max_iterations)).
+// Node pool unbounded. stats as in orc_uct_search. Returns the chosen move
+// (max visits, lowest index on ties; -1 terminal).
 int orc_mcts_timed(const orc_position* root, int nthreads, double budget_ms, uint64_t seed,
-                   double C, int64_t* stats) {
+                   double C, int64_t* stats, uint64_t max_iterations) {
   for (int i = 0; i < 199; ++i) stats[i] = 0;
   uint64_t own, opp;
   to_own_opp(*root, &own, &opp);
   Node r0 = make_node(own, opp, -1, -1);
   if (r0.terminal) return -1;
+  if (budget_ms <= 0.0 && max_iterations == 0) return -1;
   int T = resolve_threads(nthreads);
   auto t0 = std::chrono::steady_clock::now();
   auto deadline = t0 + std::chrono::duration<double, std::milli>(budget_ms);
+  const uint64_t cap = max_iterations ? max_iterations : ~0ULL;
   std::vector<TreeResult> res(T);
+  std::vector<uint64_t> plies(T, 0);
   auto worker = [&](int tid) {
-    // Grow iterations in chunks (table sized as we go) until the deadline.
-    std::vector<double> lnT(1);
-    lnT[0] = 0.0;
+    // ln table for unit 1 (lnT[k] = RN(ln k)), extended as the tree grows
+    std::vector<double> lnT(1, 0.0);
     TreeResult& tr = res[tid];
     tr.nodes.clear();
     tr.nodes.push_back(make_node(own, opp, -1, -1));
     uint64_t it = 0;
-    while (std::chrono::steady_clock::now() < deadline) {
-      uint64_t chunk = 64;
+    while (it < cap && (budget_ms <= 0.0 || std::chrono::steady_clock::now() < deadline)) {
+      uint64_t chunk = std::min<uint64_t>(64, cap - it);  // deadline checked every 64 iterations
       size_t need = it + chunk + 2;
       if (lnT.size() < need) {
         size_t old = lnT.size();
         lnT.resize(need * 2);
         for (size_t k = old; k < lnT.size(); ++k) lnT[k] = ln_rn(k);
       }
-      // Continue the same tree: run `chunk` more iterations with ids it..it+chunk-1.
-      std::vector<Node>& nodes = tr.nodes;
-      for (uint64_t j = 0; j < chunk; ++j, ++it) {
-        std::vector<int> path;
-        int v = 0;
-        path.push_back(v);
-        while (!nodes[v].terminal && fully_expanded(nodes[v])) {
-          const Node& p = nodes[v];
-          double lp = lnT[p.n];
-          int best = -1;
-          double bu = -INFINITY;
-          for (int c : p.children) {
-            double u = ucb(nodes[c].w, nodes[c].n, lp, C);
-            if (u > bu) { bu = u; best = c; }
-          }
-          v = best;
-          path.push_back(v);
-        }
-        if (!nodes[v].terminal) {
-          const Node& p = nodes[v];
-          int mv;
-          uint64_t cown, copp;
-          if (p.legal_moves == 0) { mv = 64; cown = p.opp; copp = p.own; }
-          else {
-            int idx = (int)p.children.size(), seen = 0;
-            mv = -1;
-            for (int s = 0; s < 64; ++s)
-              if ((p.legal_moves >> s) & 1) { if (seen == idx) { mv = s; break; } ++seen; }
-            uint64_t f = flips(p.own, p.opp, mv);
-            cown = p.opp & ~f; copp = p.own | f | (1ULL << mv);
-          }
-          nodes.push_back(make_node(cown, copp, mv, v));
-          int c = (int)nodes.size() - 1;
-          nodes[v].children.push_back(c);
-          v = c;
-          path.push_back(v);
-        }
-        uint64_t wins = 0, draws = 0, losses = 0;
-        const Node& leaf = nodes[v];
-        if (leaf.terminal) {
-          int a = popcount64(leaf.own), b = popcount64(leaf.opp);
-          if (a > b) wins = 1; else if (a == b) draws = 1; else losses = 1;
-        } else {
-          int rr = playout(leaf.own, leaf.opp, seed, (uint32_t)tid, (uint32_t)it, 0u, nullptr);
-          if (rr > 0) wins = 1; else if (rr == 0) draws = 1; else losses = 1;
-        }
-        uint64_t mw = losses, ow = wins;
-        for (int i = (int)path.size() - 1; i >= 0; --i) {
-          Node& x = nodes[path[i]];
-          x.n += 1; x.w += mw; x.d += draws;
-          std::swap(mw, ow);
-        }
-      }
+      for (uint64_t j = 0; j < chunk; ++j, ++it)
+        uct_iteration(&tr, it, 1u, seed, (uint32_t)tid, C, ~0ULL, lnT, &plies[tid]);
     }
     tr.iterations = it;
   };
@@ -649,9 +619,11 @@ int orc_mcts_timed(const orc_position* root, int nthreads, double budget_ms, uin
     }
     stats[195] += (int64_t)nodes[0].n;
     stats[196] += (int64_t)res[t].iterations;
+    stats[197] += (int64_t)plies[t];
+    stats[198] += (int64_t)res[t].depth_sum;
   }
   int best = -1;
-  int64_t bv = -1;
+  int64_t bv = 0;
   for (int mv = 0; mv < 65; ++mv)
     if (stats[mv] > bv) { bv = stats[mv]; best = mv; }
   return best;

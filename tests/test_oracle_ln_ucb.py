@@ -79,3 +79,49 @@ def test_ucb_terms_are_distinguishable(orc):
     assert orc.ucb(0, 4, 16.0, 1.0) == 2.0
     assert orc.ucb(0, 4, 16.0, 0.5) == 1.0
     assert orc.ucb(2, 4, 16.0, 1.0) == 2.5
+
+
+def _ucb_r1(w, n, lnT, C):
+    """Reading R1's operation order, each step an IEEE double RN operation
+    (Python floats): exploit = w/n; ratio = lnT/n; root = sqrt(ratio);
+    explore = C*root; u = exploit + explore."""
+    exploit = float(w) / float(n)
+    root = math.sqrt(lnT / float(n))
+    return exploit + C * root
+
+
+def _alternatives(w, n, lnT, C):
+    """Plausible mis-orderings of the same formula, each correctly rounded per step."""
+    from fractions import Fraction
+    exploit = float(w) / float(n)
+    root = math.sqrt(lnT / float(n))
+    return {
+        "sqrt(lnT)/sqrt(n)": exploit + C * (math.sqrt(lnT) / math.sqrt(float(n))),
+        "C*sqrt(lnT)/sqrt(n)": exploit + (C * math.sqrt(lnT)) / math.sqrt(float(n)),
+        "fma(C, root, exploit)": float(Fraction(C) * Fraction(root) + Fraction(exploit)),
+        "sqrt(C*C*lnT/n)": exploit + math.sqrt(C * C * lnT / float(n)),
+        "(w + C*sqrt(lnT*n))/n": (float(w) + C * math.sqrt(lnT * float(n))) / float(n),
+    }
+
+
+def test_ucb_operation_order_pinned(orc):
+    """The oracle's UCB is R1's five RN operations in R1's order, bit for bit,
+    and each plausible re-ordering differs from it on some of these inputs (so
+    the test would catch the slip, which the 4-ulp bound above cannot)."""
+    rng = random.Random(17)
+    differs = {}
+    for _ in range(20000):
+        unit = rng.choice([1, 32, 64, 128, 16384])
+        n = unit * rng.randrange(1, 5000)
+        w = rng.randrange(0, n + 1)
+        T = n + unit * rng.randrange(1, 50000)
+        C = rng.choice([0.25, 0.5, 1.0 / 3.0, math.sqrt(2), 0.7, 1.5])
+        lnT = rn_ln(T)
+        got = orc.ucb(w, n, lnT, C)
+        want = _ucb_r1(w, n, lnT, C)
+        assert got == want, (w, n, T, C)
+        for name, alt in _alternatives(w, n, lnT, C).items():
+            if alt != want:
+                differs[name] = differs.get(name, 0) + 1
+    for name in _alternatives(1, 2, 1.0, 1.0):
+        assert differs.get(name, 0) >= 20, (name, differs)

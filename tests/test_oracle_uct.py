@@ -176,3 +176,50 @@ def test_depth_sum_equals_tree_visits(orc, seed, unit, iters, cap):
         s, _, _ = orc.uct_search(root, 1, unit, iters, seed, tree_id_base=seed, capacity=cap)
         t = orc.uct_tree(root, unit, iters, seed, tree_id=seed, C=1.0, capacity=cap)
         assert int(s[198]) == sum(int(x) for x in t["n"][1:]) // unit
+
+
+# ---------------------------------------------------------------- the CPU opponent
+@pytest.mark.parametrize("threads,iters,seed,C,lmin,lmax", [
+    (1, 300, 3, 1.0, 0, 0),      # the opening
+    (4, 200, 5, 0.25, 20, 40),   # the C the self-play runs use
+    (3, 150, 7, 2.0, 40, 50),    # late game: passes and terminal nodes in the tree
+    (16, 64, 9, 0.0, 10, 30),    # pure exploitation
+])
+def test_mcts_timed_capped_equals_uct_search(orc, threads, iters, seed, C, lmin, lmax):
+    """The root-parallel CPU opponent, capped at `iters`
+    iterations per thread with no deadline, is T independent unit-1 trees keyed
+    (c0 = thread, c1 = iteration, c2 = 0) summed at the root: bit for bit
+    uct_search(root, T, 1, iters, seed) — all 199 stats and the move."""
+    root = orc.gen_positions(seed, 1, lmin, lmax) if lmax else orc.opening()
+    got, best = orc.mcts_timed(root, threads, 0.0, seed, C=C, max_iterations=iters)
+    want, wbest, plies = orc.uct_search(root, threads, 1, iters, seed, C=C)
+    assert got.tolist() == want.tolist()
+    assert best == wbest
+    assert got[196] == threads * iters and got[195] == threads * iters and got[197] == plies
+
+
+def test_mcts_timed_cap_with_generous_deadline(orc):
+    """A deadline that does not bind changes nothing."""
+    root = orc.gen_positions(11, 1, 20, 30)
+    got, best = orc.mcts_timed(root, 2, 60000.0, 4, C=0.5, max_iterations=100)
+    want, wbest, _ = orc.uct_search(root, 2, 1, 100, 4, C=0.5)
+    assert got.tolist() == want.tolist() and best == wbest
+
+
+def test_mcts_timed_time_mode_invariants(orc):
+    """Time mode (the self-play opponent): one playout per iteration, root
+    visits = iterations = sum of root-child visits, legal best move = argmax."""
+    root = orc.gen_positions(12, 1, 10, 30)
+    s, best = orc.mcts_timed(root, 4, 60.0, 5, C=0.25)
+    assert s[196] >= 4 and s[195] == s[196] == s[:65].sum()
+    assert (s[65:130] + s[130:195] <= s[:65]).all()
+    own, opp = own_opp(root)
+    assert (orc.legal(own, opp) >> best) & 1
+    assert best == int(np.argmax(s[:65]))
+
+
+def test_mcts_timed_terminal_root(orc):
+    full_black = (1 << 40) - 1
+    s, best = orc.mcts_timed(orc.position(full_black, ((1 << 64) - 1) & ~full_black, 0), 2, 0.0, 1,
+                             max_iterations=10)
+    assert best == -1 and (s == 0).all()
