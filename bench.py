@@ -26,7 +26,7 @@ import tempfile
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
-STATS_LEN = 199  # include/mcts.h MCTS_STATS_LEN
+STATS_LEN = 202  # include/mcts.h MCTS_STATS_LEN
 sys.path.insert(0, ROOT)
 
 N_LEAVES, N_PER_LEAF, GEN_SEED, LMIN, LMAX = 4096, 256, 2, 20, 40
@@ -50,18 +50,61 @@ METRIC = "8x8 Reversi playouts/sec at 1/2/4/8 B200; win% vs CPU-oracle MCTS"
 ALG_OPS_PER_PLY = 440
 
 
+def kernel_source_hash() -> str:
+    """sha256 (16 hex) of the sources and flags the playout kernel is built from;
+    stored with each committed ncu capture so a stale capture is detected."""
+    import hashlib
+    from paper_conf_ipps_rockis11_b200 import _build
+    h = hashlib.sha256()
+    for name in ("reversi_device.cuh", "kernels.cuh"):
+        h.update(open(os.path.join(_build.CSRC, name), "rb").read())
+    h.update(" ".join(_build.NVCC_FLAGS).encode())
+    return h.hexdigest()[:16]
+
+
 def ops_per_ply(kernel="playouts", plies_per_launch=None):
-    """(thread-instructions per ply, basis) for the roofline numerator: ncu
-    smsp__thread_inst_executed (= inst_executed x lanes active) of the committed
-    --set full capture of this kernel (profiles/latest_ncu.json), divided by the
-    plies of one launch of the same workload."""
+    """(thread-instructions per ply, basis) for the executed-instruction
+    roofline: ncu smsp__thread_inst_executed (= inst_executed x lanes active) of
+    the committed --set full capture of this kernel (profiles/latest_ncu.json),
+    divided by the plies of one launch of the same workload. If the capture was
+    taken from other kernel sources (source hash mismatch) or is missing, the
+    SURVEY.md 8(d) model is used and the basis says so (with a warning)."""
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))[kernel]
+        if prof.get("source_hash") != kernel_source_hash():
+            print(f"[bench] warning: profiles/latest_ncu.json {kernel} capture is stale "
+                  f"(source hash {prof.get('source_hash')} != {kernel_source_hash()}); "
+                  "using the SURVEY 8(d) model", file=sys.stderr)
+            return ALG_OPS_PER_PLY, "model: SURVEY.md 8(d) estimate (committed capture is stale)"
         plies = plies_per_launch or prof["plies_per_launch"]
         return prof["thread_inst"] / plies, ("measured: ncu smsp__thread_inst_executed.sum / plies, "
-                                             f"committed capture of {kernel}_kernel (profiles/latest_ncu.json)")
+                                             f"committed capture of {kernel}_kernel (profiles/latest_ncu.json, "
+                                             f"source hash {prof['source_hash']})")
     except Exception:
         return ALG_OPS_PER_PLY, "model: SURVEY.md 8(d) estimate (no committed capture)"
+
+
+def headline(playouts_total, plies_total, t_ms_max, steps):
+    """The line's throughput numbers from whole-job counts and the max-over-ranks
+    device time of the `steps` timed steps."""
+    s = t_ms_max / 1e3
+    return {"value": playouts_total / s, "plies_per_s": plies_total / s, "ms_per_step": t_ms_max / steps}
+
+
+def roofline(plies_per_launch, kern_s, peak_ops, ops_exec, ops_basis, alu_peak, peak_basis):
+    """The integer roofline of the playout kernel, both ways:
+    frac = SURVEY.md 8(d)'s algorithmic ops per ply (ALG_OPS_PER_PLY) x plies per
+    launch / launch time / peak (the contract's ALGORITHMIC numerator; > 1 means
+    the kernel needs fewer instructions than the model); frac_executed = the
+    executed thread-instructions per ply (ncu) x plies / time / peak, i.e. the
+    share of the chip's integer issue rate the kernel keeps busy."""
+    alg = plies_per_launch * ALG_OPS_PER_PLY / kern_s
+    exe = plies_per_launch * ops_exec / kern_s
+    return {"bound": "alu", "achieved": alg / 1e9, "peak": peak_ops / 1e9, "unit": "Gop/s",
+            "frac": alg / peak_ops, "frac_basis": f"algorithmic: SURVEY.md 8(d) {ALG_OPS_PER_PLY} int ops per ply",
+            "achieved_executed": exe / 1e9, "frac_executed": exe / peak_ops, "ops_per_ply_executed": ops_exec,
+            "ops_basis": ops_basis, "plies_per_launch": plies_per_launch, "peak_basis": peak_basis,
+            "alu_pipe_peak": alu_peak / 1e9}
 
 
 def clocks_sampler(path):
@@ -154,8 +197,9 @@ def reference_arm(args, rank):
     }), flush=True)
 
 
-def cpu_baseline(budget_s=12.0):
-    """The oracle timed on the host cores on a bounded sample of configs[1]."""
+def cpu_baseline(budget_s=12.0, single_budget_s=4.0):
+    """The oracle timed on the host cores on a bounded sample of configs[1]:
+    all cores (the reported value) and one core (`single_core`)."""
     import oracle
     cores = len(os.sched_getaffinity(0))
     leaves = oracle.gen_positions(GEN_SEED, N_LEAVES, LMIN, LMAX)
@@ -165,8 +209,15 @@ def cpu_baseline(budget_s=12.0):
                         nthreads=cores)
         done += 128
     dt = time.perf_counter() - t0
+    one, t1 = 0, time.perf_counter()
+    while one < N_LEAVES and time.perf_counter() - t1 < single_budget_s:
+        oracle.playouts(leaves[one:one + 2], N_PER_LEAF, PLAYOUT_SEED, leaf_id_base=one, nthreads=1)
+        one += 2
+    d1 = time.perf_counter() - t1
     return {"value": done * N_PER_LEAF / dt, "unit": "playouts/s", "cores": cores, "kind": "oracle",
-            "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)"}
+            "sample": f"leaves 0..{done - 1} of configs[1] x {N_PER_LEAF} playouts ({dt:.1f} s)",
+            "single_core": {"value": one * N_PER_LEAF / d1, "cores": 1,
+                            "sample": f"leaves 0..{one - 1} of configs[1] x {N_PER_LEAF} playouts ({d1:.1f} s)"}}
 
 
 def sweep_leg(args, local):
@@ -344,7 +395,7 @@ def selfplay_leg(args, world, rank, local):
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_rockis11_b200 as pkg
-    from paper_conf_ipps_rockis11_b200.distributed import merge_root_stats, best_move_from
+    from paper_conf_ipps_rockis11_b200.distributed import merge_root_stats
 
     torch.cuda.set_device(local)
     if world > 1:
@@ -371,7 +422,7 @@ def selfplay_leg(args, world, rank, local):
             merge_root_stats(stats)
         torch.cuda.synchronize()
         st = stats.cpu().numpy()
-        return best_move_from(st), int(st[195]), float(st[198]) / max(int(st[196]), 1)
+        return pkg.best_move(st), int(st[195]), float(st[198]) / max(int(st[196]), 1)
 
     if rank != 0:  # follower ranks: search whatever position rank 0 broadcasts
         while True:
@@ -422,13 +473,40 @@ def selfplay_leg(args, world, rank, local):
         dist.destroy_process_group()
 
 
+def self_launch_cmd(gpus, argv, env):
+    """`python bench.py --gpus N` outside torchrun: the torchrun command that runs
+    this script as N ranks (one per GPU, rendezvous on 127.0.0.1), or None when
+    already under torchrun or N == 1. Under torchrun WORLD_SIZE must equal N."""
+    if "WORLD_SIZE" in env:
+        if int(env["WORLD_SIZE"]) != gpus:
+            raise SystemExit(f"bench.py: --gpus {gpus} but WORLD_SIZE={env['WORLD_SIZE']}")
+        return None
+    if gpus <= 1:
+        return None
+    import socket
+    with socket.socket() as sk:  # a free rendezvous port
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *argv]
+
+
 def init_dist(dist, torch, local):
-    """One process per GPU over NCCL (BENCH_BACKEND=gloo is a single-GPU test hook)."""
+    """One process per GPU over NCCL (BENCH_BACKEND=gloo is a single-GPU test hook).
+    Logs the communicator (backend, rank, world size, device) on stderr."""
     backend = os.environ.get("BENCH_BACKEND", "nccl")
     if backend == "nccl":
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     else:
         dist.init_process_group(backend)
+    print(f"[bench] process group: backend={dist.get_backend()} rank={dist.get_rank()} "
+          f"world={dist.get_world_size()} device=cuda:{local}", file=sys.stderr, flush=True)
+
+
+def pool_info(st) -> dict:
+    """Node-pool saturation of a search (stats [199]-[201], include/mcts.h)."""
+    return {"refused_expansions": int(st[199]), "pool_slots_used": int(st[200]),
+            "pool_slot_capacity": int(st[201])}
 
 
 def log(*a):
@@ -473,6 +551,9 @@ def main():
                     help="iteration-mode search legs (profiling); default: time mode")
     args = ap.parse_args()
 
+    cmd = self_launch_cmd(args.gpus, sys.argv[1:], os.environ)
+    if cmd is not None:  # --gpus N without torchrun: one process per GPU, launched here
+        sys.exit(subprocess.call(cmd))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -554,8 +635,7 @@ def main():
     t_ms = max_over_ranks(kernel_ms)
     plies_total = sum_over_ranks(plies_local)
     playouts_total = world * args.steps * N_LEAVES * N_PER_LEAF
-    value = playouts_total / (t_ms / 1e3)
-    ms_per_step = t_ms / args.steps
+    head = headline(playouts_total, plies_total, t_ms, args.steps)
 
     log('# ---- end to end')
     # ---- end to end through the C ABI with host buffers (H2D + kernel + D2H)
@@ -640,7 +720,7 @@ def main():
             "iterations_per_tree": float(st[196]) / (SEARCH_TREES * world),
             "plies_per_s": float(st[197]) / (s_ms / 1e3),
             "best_move": int(pkg.best_move(st)), "allreduce": world > 1,
-            "mean_depth": float(st[198]) / max(float(st[196]), 1.0),
+            "mean_depth": float(st[198]) / max(float(st[196]), 1.0), **pool_info(st),
             # the playout kernel's measured instructions per ply (the search
             # kernel's playouts run the same loop), per GPU
             "roofline_frac": float(st[197]) / world / (s_ms / 1e3) * ops_per_ply("playouts")[0]
@@ -654,17 +734,19 @@ def main():
             "playouts_per_s": float(lt[195]) / (l_ms / 1e3), "ms": l_ms,
             "iterations": float(lt[196]) / world, "plies_per_s": float(lt[197]) / (l_ms / 1e3),
             "best_move": int(pkg.best_move(lt)), "mean_depth": float(lt[198]) / max(float(lt[196]), 1.0),
+            **pool_info(lt),
         }
         ml.close()
         log('mt = pkg.Mcts(')
         mt = pkg.Mcts(c_uct=1.0, scheme="tree", device=local)
-        tt, t_ms = run_search(mt, SEARCH_TREES, SEARCH_THREADS, rank, it_scale=SEARCH_TREES)
+        tt, tree_ms = run_search(mt, SEARCH_TREES, SEARCH_THREADS, rank, it_scale=SEARCH_TREES)
         tree_search = {
             "workload": f"NEXT-4 tree parallelism: one shared tree, {SEARCH_TREES} workers x {SEARCH_THREADS} "
                         f"threads per GPU, {mode}, opening root, C=1.0",
-            "playouts_per_s": float(tt[195]) / (t_ms / 1e3), "ms": t_ms,
-            "iterations": float(tt[196]) / world, "plies_per_s": float(tt[197]) / (t_ms / 1e3),
+            "playouts_per_s": float(tt[195]) / (tree_ms / 1e3), "ms": tree_ms,
+            "iterations": float(tt[196]) / world, "plies_per_s": float(tt[197]) / (tree_ms / 1e3),
             "best_move": int(pkg.best_move(tt)), "mean_depth": float(tt[198]) / max(float(tt[196]), 1.0),
+            **pool_info(tt),
         }
         mt.close()
 
@@ -684,18 +766,22 @@ def main():
     kern_s = kernel_ms / 1e3 / args.steps
     plies_per_launch = plies_local / args.steps
     opp, opp_basis = ops_per_ply("playouts", plies_per_launch)
-    achieved = plies_per_launch * opp / kern_s
+    roof = roofline(plies_per_launch, kern_s, peak_ops, opp, opp_basis, alu_peak, peak_basis)
     traffic, ncu = None, None
     try:  # from the committed ncu --set full capture of this kernel (profiles/latest_ncu.json)
         prof = json.load(open(os.path.join(ROOT, "profiles", "latest_ncu.json")))["playouts"]
-        traffic = prof["dram_bytes_per_launch"]
-        ncu = {k: prof.get(k) for k in ("alu_pipe_pct", "fmaheavy_pipe_pct", "issue_active_pct",
-                                        "lanes_active_per_inst", "thread_inst", "duration_us")}
+        if prof.get("source_hash") == kernel_source_hash():
+            traffic = prof["dram_bytes_per_launch"]
+            ncu = {k: prof.get(k) for k in ("alu_pipe_pct", "fmaheavy_pipe_pct", "issue_active_pct",
+                                            "lanes_active_per_inst", "thread_inst", "duration_us",
+                                            "source_hash", "capture")}
     except Exception:
         pass
+    roof["traffic"] = traffic
+    roof["ncu"] = ncu
     line = {
-        "metric": METRIC, "value": value, "unit": "playouts/s", "n_gpus": world,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+        "metric": METRIC, "value": head["value"], "unit": "playouts/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
         "data": "synthetic",
         "config": {"workload": "configs[1]: 4096 synthetic mid-game positions (seed 2, 20-40 random "
@@ -703,13 +789,8 @@ def main():
                    "global_batch": world * N_LEAVES * N_PER_LEAF,
                    "parallelism": f"leaf-range x{world} (weak)",
                    "l2": "flushed between steps (256 MiB write outside the timed events)"},
-        "plies_per_s": plies_total / (t_ms / 1e3),
-        "roofline": {"bound": "alu", "achieved": achieved / 1e9, "peak": peak_ops / 1e9,
-                     "unit": "Gop/s", "frac": achieved / peak_ops, "traffic": traffic,
-                     "ops_per_ply": opp, "ops_basis": opp_basis, "plies_per_launch": plies_per_launch,
-                     "ncu": ncu, "peak_basis": peak_basis, "alu_pipe_peak": alu_peak / 1e9,
-                     "survey_model": {"ops_per_ply": ALG_OPS_PER_PLY,
-                                      "frac": plies_per_launch * ALG_OPS_PER_PLY / kern_s / peak_ops}},
+        "plies_per_s": head["plies_per_s"],
+        "roofline": roof,
         "e2e": {"value": e2e_value, "unit": "playouts/s",
                 "h2d_bytes_per_step": N_LEAVES * 24, "d2h_bytes_per_step": N_LEAVES * 12 + 8,
                 "api": "mcts_playouts (host buffers, pinned)"},

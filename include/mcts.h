@@ -81,7 +81,9 @@ typedef struct {
 typedef struct {
   double c_uct;                /* UCB exploration constant C (L169); finite, >= 0; R1 default 1.0 */
   uint32_t scheme;             /* MCTS_BLOCK, MCTS_LEAF or MCTS_TREE */
-  uint32_t max_nodes_per_tree; /* time mode: node-slot pool per tree (0 = 65536; MCTS_TREE: 2^26) */
+  uint32_t max_nodes_per_tree; /* time mode: node-slot pool per tree; 0 = sized from the
+                                  time budget and free HBM (stats [199]-[201]
+                                  report refusals and use) */
   int32_t device;              /* CUDA device ordinal */
   uint32_t flags;              /* 0 or MCTS_FLAG_CHECK_TREE; other bits: INVALID_ARGUMENT */
 } mcts_params;
@@ -104,8 +106,17 @@ typedef struct {
  *   [197]     playout plies (non-pass moves simulated)
  *   [198]     sum over iterations of the simulated node's depth (edges
  *             from the root; mean tree depth = [198] / [196], the paper's
- *             "Depth" of Fig. 8)                               */
-#define MCTS_STATS_LEN 199
+ *             "Depth" of Fig. 8)
+ *   [199]     iterations whose expansion was refused because the tree's node
+ *             pool was full (time mode only; "I add one node per iteration",
+ *             L179-L182, cannot hold then: the selected node is simulated
+ *             again, R12). 0 in iteration mode.
+ *   [200]     node-pool slots used (summed over trees; a node reserves its
+ *             whole child block at its first expansion)
+ *   [201]     node-pool slot capacity (summed over trees)
+ * [0,200) are bit-exact to the oracle in iteration mode; [200] and [201]
+ * describe this library's pools (the oracle counts nodes, not slots). */
+#define MCTS_STATS_LEN 202
 
 typedef struct {
   uint64_t visits[65];
@@ -115,6 +126,9 @@ typedef struct {
   uint64_t iterations_done;
   uint64_t plies;
   uint64_t depth_sum; /* [198]: sum over iterations of the simulated node's depth */
+  uint64_t refused_expansions; /* [199]: expansions refused by a full node pool */
+  uint64_t slots_used;         /* [200] */
+  uint64_t slot_capacity;      /* [201] */
   int32_t best_move; /* argmax visits, lowest index on ties (R8); -1 if the root is terminal */
   int32_t reserved;
 } mcts_root_stats;

@@ -23,7 +23,7 @@ LIB = os.path.join(HERE, "liboracle.so")
 POSITION_DTYPE = np.dtype(
     [("black", "<u8"), ("white", "<u8"), ("to_move", "<u4"), ("reserved", "<u4")]
 )
-N_STATS = 199
+N_STATS = 202
 
 
 def build(force: bool = False) -> str:
@@ -152,8 +152,9 @@ def ucb(w: int, n: int, ln_parent: float, C: float) -> float:
 
 def uct_search(root: np.ndarray, n_trees: int, unit: int, iterations: int, seed: int,
                tree_id_base: int = 0, C: float = 1.0, capacity: int = 0, nthreads: int = 0):
-    """UCT search (PAPER.md L155-L202), iteration mode. Returns (stats[199], best, plies);
-    stats[197] = plies, stats[198] = sum over iterations of the simulated node's depth."""
+    """UCT search (PAPER.md L155-L202), iteration mode. Returns (stats[202], best, plies);
+    stats[197] = plies, stats[198] = sum over iterations of the simulated node's depth,
+    [199] expansions refused by a full pool, [200] nodes, [201] node capacity (summed)."""
     stats = np.zeros(N_STATS, dtype=np.int64)
     plies = ctypes.c_uint64(0)
     best = lib().orc_uct_search(_ptr(root), n_trees, unit, iterations, seed, tree_id_base, C,

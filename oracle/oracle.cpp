@@ -240,6 +240,7 @@ struct TreeResult {
   std::vector<Node> nodes;
   uint64_t iterations = 0;
   uint64_t depth_sum = 0;  // sum over iterations of the simulated node's depth (edges from the root)
+  uint64_t refused = 0;    // iterations whose expansion the full node pool refused (R12)
 };
 
 // One UCT iteration (number `it`) on a tree whose root is nodes[0], with `unit`
@@ -293,6 +294,8 @@ void uct_iteration(TreeResult* out, uint64_t it, uint32_t unit, uint64_t seed, u
     nodes[v].children.push_back(c);
     v = c;
     path.push_back(v);
+  } else if (!nodes[v].terminal) {
+    out->refused += 1;  // pool full: simulate from the selected node itself (R12)
   }
   // 3) Simulation (L183-L195): `unit` playouts from the leaf.
   uint64_t wins = 0, draws = 0, losses = 0;  // for the leaf's side to move
@@ -440,14 +443,15 @@ double orc_ucb(uint64_t w, uint64_t n, double ln_parent, double C) { return ucb(
 // Full search (the mcts_search contract, iteration mode). stats layout:
 // [0,65) visits, [65,130) wins (for the root's side to move), [130,195) draws,
 // [195] root visits, [196] iterations, [197] playout plies, [198] sum over
-// iterations of the simulated node's depth; summed over trees tree_id_base ..
+// iterations of the simulated node's depth, [199] expansions refused by a full
+// pool, [200] nodes, [201] node capacity; summed over trees tree_id_base ..
 // tree_id_base + n_trees - 1. capacity = max nodes per tree (0 = iterations+1).
 // Returns best move (max visits, lowest index on ties) or -1 if the root is
 // terminal. plies_out (nullable) receives the playout plies.
 int orc_uct_search(const orc_position* root, uint32_t n_trees, uint32_t unit, uint64_t iterations,
                    uint64_t seed, uint32_t tree_id_base, double C, uint64_t capacity,
                    int64_t* stats, uint64_t* plies_out, int nthreads) {
-  for (int i = 0; i < 199; ++i) stats[i] = 0;
+  for (int i = 0; i < 202; ++i) stats[i] = 0;
   uint64_t own, opp;
   to_own_opp(*root, &own, &opp);
   if (capacity == 0) capacity = iterations + 1;
@@ -481,6 +485,11 @@ int orc_uct_search(const orc_position* root, uint32_t n_trees, uint32_t unit, ui
     stats[195] += (int64_t)nodes[0].n;
     stats[196] += (int64_t)res[t].iterations;
     stats[198] += (int64_t)res[t].depth_sum;
+    stats[199] += (int64_t)res[t].refused;
+    if (!nodes[0].terminal) {  // a terminal root is no search: all stats stay 0
+      stats[200] += (int64_t)nodes.size();
+      stats[201] += (int64_t)capacity;
+    }
     ptot += plies[t];
   }
   stats[197] = (int64_t)ptot;
@@ -573,7 +582,7 @@ void orc_gen_positions(uint64_t seed, uint32_t n, uint32_t lmin, uint32_t lmax, 
 // (max visits, lowest index on ties; -1 terminal).
 int orc_mcts_timed(const orc_position* root, int nthreads, double budget_ms, uint64_t seed,
                    double C, int64_t* stats, uint64_t max_iterations) {
-  for (int i = 0; i < 199; ++i) stats[i] = 0;
+  for (int i = 0; i < 202; ++i) stats[i] = 0;
   uint64_t own, opp;
   to_own_opp(*root, &own, &opp);
   Node r0 = make_node(own, opp, -1, -1);
@@ -621,6 +630,7 @@ int orc_mcts_timed(const orc_position* root, int nthreads, double budget_ms, uin
     stats[196] += (int64_t)res[t].iterations;
     stats[197] += (int64_t)plies[t];
     stats[198] += (int64_t)res[t].depth_sum;
+    stats[200] += (int64_t)nodes.size();
   }
   int best = -1;
   int64_t bv = 0;

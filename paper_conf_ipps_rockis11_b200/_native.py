@@ -16,7 +16,7 @@ POSITION_DTYPE = np.dtype(
     [("black", "<u8"), ("white", "<u8"), ("to_move", "<u4"), ("reserved", "<u4")]
 )
 WDL_DTYPE = np.dtype([("wins", "<u4"), ("draws", "<u4"), ("losses", "<u4")])
-STATS_LEN = 199
+STATS_LEN = 202
 MCTS_BLOCK, MCTS_LEAF, MCTS_TREE = 0, 1, 2
 MCTS_FLAG_CHECK_TREE = 1
 
@@ -53,7 +53,9 @@ class RootStats(ctypes.Structure):
     _fields_ = [("visits", ctypes.c_uint64 * 65), ("wins", ctypes.c_uint64 * 65),
                 ("draws", ctypes.c_uint64 * 65), ("root_visits", ctypes.c_uint64),
                 ("iterations_done", ctypes.c_uint64), ("plies", ctypes.c_uint64),
-                ("depth_sum", ctypes.c_uint64), ("best_move", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("depth_sum", ctypes.c_uint64), ("refused_expansions", ctypes.c_uint64),
+                ("slots_used", ctypes.c_uint64), ("slot_capacity", ctypes.c_uint64),
+                ("best_move", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 _lib = None
@@ -185,15 +187,7 @@ class Mcts:
         rp = ctypes.byref(_pos(root)) if root is not None else None
         self._check(self.L.mcts_search(self.h, rp, Budget(iterations, time_ms), n_trees,
                                        threads_per_tree, seed, ctypes.byref(out)))
-        stats = np.zeros(STATS_LEN, dtype=np.int64)
-        stats[0:65] = np.ctypeslib.as_array(out.visits)
-        stats[65:130] = np.ctypeslib.as_array(out.wins)
-        stats[130:195] = np.ctypeslib.as_array(out.draws)
-        stats[195], stats[196], stats[197] = out.root_visits, out.iterations_done, out.plies
-        stats[198] = out.depth_sum
-        return dict(stats=stats, best_move=int(out.best_move), root_visits=int(out.root_visits),
-                    iterations=int(out.iterations_done), plies=int(out.plies),
-                    depth_sum=int(out.depth_sum))
+        return self._stats_dict(out)
 
     @staticmethod
     def _stats_dict(out: "RootStats") -> dict:
@@ -202,10 +196,12 @@ class Mcts:
         stats[65:130] = np.ctypeslib.as_array(out.wins)
         stats[130:195] = np.ctypeslib.as_array(out.draws)
         stats[195], stats[196], stats[197] = out.root_visits, out.iterations_done, out.plies
-        stats[198] = out.depth_sum
+        stats[198], stats[199] = out.depth_sum, out.refused_expansions
+        stats[200], stats[201] = out.slots_used, out.slot_capacity
         return dict(stats=stats, best_move=int(out.best_move), root_visits=int(out.root_visits),
                     iterations=int(out.iterations_done), plies=int(out.plies),
-                    depth_sum=int(out.depth_sum))
+                    depth_sum=int(out.depth_sum), refused_expansions=int(out.refused_expansions),
+                    slots_used=int(out.slots_used), slot_capacity=int(out.slot_capacity))
 
     def search_hybrid(self, root=None, iterations: int = 0, time_ms: float = 0.0, n_trees: int = 1,
                       threads_per_tree: int = 64, seed: int = 1, cpu_threads: int = 1) -> dict:

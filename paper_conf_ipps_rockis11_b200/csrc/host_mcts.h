@@ -24,7 +24,7 @@ struct HostSearchArgs {
   const double* lnT;           // lnT[k] = RN(ln k), k <= iterations (from the device ln table)
 };
 
-// Runs the host trees; writes MCTS_STATS_LEN (199) int64 sums into stats.
+// Runs the host trees; writes MCTS_STATS_LEN (202) int64 sums into stats.
 void search(const HostSearchArgs& a, int64_t* stats);
 
 }  // namespace mcts_host

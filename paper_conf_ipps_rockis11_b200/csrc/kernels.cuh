@@ -155,6 +155,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
   u32 plies = 0;
   u32 it = 0;
   unsigned long long depth_sum = 0;  // lane 0 of warp 0: sum of leaf depths (Fig. 8 "Depth")
+  unsigned long long refused = 0;    // lane 0 of warp 0: expansions refused by a full pool
   if (!meta_term(T.meta[base])) {
     for (;; ++it) {
       if (warp == 0) {
@@ -169,6 +170,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth;
             depth_sum += (unsigned)L.depth;
+            refused += L.refused;
           }
         }
         if (lane == 0) s_stop = stop;
@@ -204,6 +206,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
     for (int off = 16; off > 0; off >>= 1) P += __shfl_xor_sync(kFull, P, off);
     if (lane == 0 && P) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, P);
     if (lane == 0 && depth_sum) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
+    if (lane == 0 && !meta_term(T.meta[base])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
     merge_root(T, base, unit, it, a.stats, lane);
   }
 }
@@ -247,6 +250,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   u32 plies = 0;
   u32 it = 0;
   unsigned long long depth_sum = 0;  // leader lane 0
+  unsigned long long refused = 0;    // leader lane 0
   for (;; ++it) {
     if (leader) {
       if (it > 0) {
@@ -267,6 +271,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
         if (lane == 0) {
           s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
           depth_sum += (unsigned)L.depth;
+          refused += L.refused;
         }
       }
       if (lane == 0) S->stop = stop;
@@ -298,6 +303,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
   if (leader && lane == 0 && depth_sum)
     atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
+  if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
 

@@ -46,6 +46,7 @@ struct mcts_handle {
   // trees
   void* pool_mem = nullptr;
   size_t pool_bytes = 0;
+  uint32_t tree_clean_cap = 0;  // MCTS_TREE: slot_cap of the carving whose unused slots are clear (0: none)
 
   // ln table
   double* d_lnT = nullptr;
@@ -131,8 +132,10 @@ mcts_status ensure_pool(mcts_handle* h, uint32_t n_trees, uint32_t slot_cap, Tre
   const size_t bytes = slots * per + 8 * 256;
   if (bytes > (size_t)96 << 30)
     return fail(h, MCTS_E_OOM, "tree pool would exceed 96 GiB; lower iterations or max_nodes_per_tree");
+  void* old = h->pool_mem;
   mcts_status st = ensure(h, &h->pool_mem, &h->pool_bytes, bytes);
   if (st) return st;
+  if (h->pool_mem != old) h->tree_clean_cap = 0;
   char* p = (char*)h->pool_mem;
   auto take = [&](size_t b) { char* q = p; p += (b + 255) & ~(size_t)255; return q; };
   T->own = (u64*)take(slots * sizeof(u64));
@@ -152,6 +155,51 @@ mcts_status check_device(mcts_handle* h) {
   cudaError_t e = cudaSetDevice(h->device);
   if (e != cudaSuccess) return fail(h, MCTS_E_NO_DEVICE, std::string("cudaSetDevice: ") + cudaGetErrorString(e));
   return MCTS_OK;
+}
+
+// Time-mode default node pool per tree (params.max_nodes_per_tree == 0): an
+// upper bound on the iterations a tree runs in the budget (per tree for
+// MCTS_BLOCK / MCTS_LEAF, for the whole shared tree with MCTS_TREE) times ~10
+// slots reserved per expanded node, rounded up to a power of two, capped so the
+// pool stays within 60% of the HBM that is free (plus the pool already held).
+uint32_t auto_slot_cap(mcts_handle* h, double time_ms, uint32_t n_trees, bool shared) {
+  size_t free_b = 0, total_b = 0;
+  if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) free_b = (size_t)8 << 30;
+  const double per_ms = shared ? 20000.0 : 100.0;  // measured: ~15k/ms shared tree, ~66/ms per block tree
+  double want = time_ms * per_ms * 10.0;
+  const double hi = shared ? (double)(1u << 28) : (double)(1u << 24);
+  if (want < 65536.0) want = 65536.0;
+  if (want > hi) want = hi;
+  uint64_t cap = 1;
+  while ((double)cap < want) cap <<= 1;
+  const uint64_t per_slot = 3 * sizeof(u64) + 6 * sizeof(u32);
+  const uint64_t mem_cap = (uint64_t)((double)(free_b + h->pool_bytes) * 0.6) / ((uint64_t)n_trees * per_slot);
+  if (cap > mem_cap) cap = mem_cap;
+  if (cap < 64) cap = 64;
+  return (uint32_t)cap;
+}
+
+// CTAs of a search kernel that can be resident at once (SMs x occupancy).
+mcts_status resident_ctas(mcts_handle* h, const void* kfn, uint32_t threads, long long* out) {
+  int per_sm = 0, n_sm = 0;
+  CK(h, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, (int)threads, 0));
+  CK(h, cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, h->device));
+  *out = (long long)per_sm * n_sm;
+  return MCTS_OK;
+}
+
+const void* block_kernel_fn(uint32_t threads) {
+  if (threads <= 128) return (const void*)block_search_kernel<128, 8>;
+  if (threads <= 256) return (const void*)block_search_kernel<256, 4>;
+  if (threads <= 512) return (const void*)block_search_kernel<512, 2>;
+  return (const void*)block_search_kernel<1024, 1>;
+}
+
+const void* tree_kernel_fn(uint32_t threads) {
+  if (threads <= 128) return (const void*)tree_search_kernel<128, 8>;
+  if (threads <= 256) return (const void*)tree_search_kernel<256, 4>;
+  if (threads <= 512) return (const void*)tree_search_kernel<512, 2>;
+  return (const void*)tree_search_kernel<1024, 1>;
 }
 
 template <int MAXT, int MINB>
@@ -180,12 +228,20 @@ mcts_status tree_search_impl(mcts_handle* h, const mcts_position* rp, uint32_t w
   mcts_status st = ensure_pool(h, 1, slot_cap, &T);
   if (st) return st;
   // cleared fields: a read racing a child's creation sees meta = 0 (skipped)
-  // or k = vl = w = 0 and first = kNoChild (tree_select_expand)
-  CK(h, cudaMemsetAsync(T.meta, 0, (size_t)slot_cap * sizeof(u32), s));
-  CK(h, cudaMemsetAsync(T.k, 0, (size_t)slot_cap * sizeof(u32), s));
-  CK(h, cudaMemsetAsync(T.w, 0, (size_t)slot_cap * sizeof(u32), s));
-  CK(h, cudaMemsetAsync(T.vl, 0, (size_t)slot_cap * sizeof(u32), s));
-  CK(h, cudaMemsetAsync(T.first, 0xFF, (size_t)slot_cap * sizeof(u32), s));
+  // or k = vl = w = 0 and first = kNoChild (tree_select_expand). A new pool
+  // carving is cleared whole; after that only the slots the previous search
+  // used (tree_clear_kernel reads its allocator).
+  if (h->tree_clean_cap != slot_cap) {
+    CK(h, cudaMemsetAsync(T.meta, 0, (size_t)slot_cap * sizeof(u32), s));
+    CK(h, cudaMemsetAsync(T.k, 0, (size_t)slot_cap * sizeof(u32), s));
+    CK(h, cudaMemsetAsync(T.w, 0, (size_t)slot_cap * sizeof(u32), s));
+    CK(h, cudaMemsetAsync(T.vl, 0, (size_t)slot_cap * sizeof(u32), s));
+    CK(h, cudaMemsetAsync(T.first, 0xFF, (size_t)slot_cap * sizeof(u32), s));
+    h->tree_clean_cap = slot_cap;
+  } else {
+    tree_clear_kernel<<<4 * 148, 256, 0, s>>>(T, h->d_treesync);
+    CK(h, cudaGetLastError());
+  }
   DevPosition root;
   memcpy(&root, rp, sizeof(DevPosition));
   tree_root_kernel<<<1, 1, 0, s>>>(T, h->d_treesync, root);
@@ -199,7 +255,7 @@ mcts_status tree_search_impl(mcts_handle* h, const mcts_position* rp, uint32_t w
   else if (unit <= 512) st = launch_tree<512, 2>(h, workers, unit, T, a, s);
   else st = launch_tree<1024, 1>(h, workers, unit, T, a, s);
   if (st) return st;
-  tree_merge_kernel<<<1, 32, 0, s>>>(T, unit, a.stats);
+  tree_merge_kernel<<<1, 32, 0, s>>>(T, h->d_treesync, unit, a.stats);
   CK(h, cudaGetLastError());
   if (h->params.flags & MCTS_FLAG_CHECK_TREE) {
     tree_check_kernel<<<592, 256, 0, s>>>(T, h->d_treesync, unit, slot_cap, h->d_error);
@@ -253,8 +309,18 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
       slot_cap = (uint32_t)(need > 0x7FFFFFFFull ? 0x7FFFFFFFull : need);
     } else {
       max_it = cap_it;
-      slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree : (1u << 26);
+      mcts_status st = check_device(h);
+      if (st) return st;
+      slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree
+                                              : auto_slot_cap(h, budget.time_ms, 1, true);
       if (slot_cap < 64) slot_cap = 64;
+      // workers that cannot be resident would only start after the deadline
+      long long res = 0;
+      st = resident_ctas(h, tree_kernel_fn(threads_per_tree), threads_per_tree, &res);
+      if (st) return st;
+      if ((long long)n_trees > res)
+        return fail(h, MCTS_E_INVALID_ARGUMENT, "time mode: n_trees (workers) exceeds the co-resident CTAs (" +
+                                                    std::to_string(res) + ") for this threads_per_tree");
     }
     mcts_status st = check_device(h);
     if (st) return st;
@@ -289,8 +355,19 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
     slot_cap = (uint32_t)(need > 0xFFFFFFF0ull ? 0xFFFFFFF0ull : need);
   } else {
     max_it = kmax_counts < (1u << 20) ? kmax_counts : (1u << 20);
-    slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree : 65536u;
+    mcts_status st = check_device(h);
+    if (st) return st;
+    slot_cap = h->params.max_nodes_per_tree ? h->params.max_nodes_per_tree
+                                            : auto_slot_cap(h, budget.time_ms, n_trees, false);
     if (slot_cap < 64) slot_cap = 64;
+    if (!leaf) {  // trees that cannot be resident would only start after the deadline
+      long long res = 0;
+      st = resident_ctas(h, block_kernel_fn(threads_per_tree), threads_per_tree, &res);
+      if (st) return st;
+      if ((long long)n_trees > res)
+        return fail(h, MCTS_E_INVALID_ARGUMENT, "time mode: n_trees exceeds the co-resident CTAs (" +
+                                                    std::to_string(res) + ") for this threads_per_tree");
+    }
   }
 
   mcts_status st = check_device(h);
@@ -341,6 +418,24 @@ mcts_status search_impl(mcts_handle* h, const mcts_position* root, mcts_budget b
   void* args[] = {(void*)&T, (void*)&a, (void*)&S};
   CK(h, cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(128), args, 0, s));
   return MCTS_OK;
+}
+
+// The stats vector (include/mcts.h MCTS_STATS_LEN) as a mcts_root_stats.
+void fill_root_stats(const long long* hs, mcts_root_stats* out) {
+  for (int i = 0; i < 65; ++i) {
+    out->visits[i] = (uint64_t)hs[i];
+    out->wins[i] = (uint64_t)hs[65 + i];
+    out->draws[i] = (uint64_t)hs[130 + i];
+  }
+  out->root_visits = (uint64_t)hs[195];
+  out->iterations_done = (uint64_t)hs[196];
+  out->plies = (uint64_t)hs[197];
+  out->depth_sum = (uint64_t)hs[198];
+  out->refused_expansions = (uint64_t)hs[199];
+  out->slots_used = (uint64_t)hs[200];
+  out->slot_capacity = (uint64_t)hs[201];
+  out->best_move = mcts_best_move((const int64_t*)hs);
+  out->reserved = 0;
 }
 
 }  // namespace
@@ -529,32 +624,8 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   CK(h, cudaStreamSynchronize(h->stream));
   if (herr == 2) return fail(h, MCTS_E_CUDA, "MCTS_TREE: tree invariant check failed (MCTS_FLAG_CHECK_TREE)");
   if (herr) return fail(h, MCTS_E_CUDA, "search kernel reported an internal error");
-  for (int i = 0; i < 65; ++i) {
-    out->visits[i] = (uint64_t)hs[i];
-    out->wins[i] = (uint64_t)hs[65 + i];
-    out->draws[i] = (uint64_t)hs[130 + i];
-  }
-  out->root_visits = (uint64_t)hs[195];
-  out->iterations_done = (uint64_t)hs[196];
-  out->plies = (uint64_t)hs[197];
-  out->depth_sum = (uint64_t)hs[198];
-  out->best_move = mcts_best_move((const int64_t*)hs);
-  out->reserved = 0;
+  fill_root_stats(hs, out);
   return MCTS_OK;
-}
-
-static void fill_root_stats(const long long* hs, mcts_root_stats* out) {
-  for (int i = 0; i < 65; ++i) {
-    out->visits[i] = (uint64_t)hs[i];
-    out->wins[i] = (uint64_t)hs[65 + i];
-    out->draws[i] = (uint64_t)hs[130 + i];
-  }
-  out->root_visits = (uint64_t)hs[195];
-  out->iterations_done = (uint64_t)hs[196];
-  out->plies = (uint64_t)hs[197];
-  out->depth_sum = (uint64_t)hs[198];
-  out->best_move = mcts_best_move((const int64_t*)hs);
-  out->reserved = 0;
 }
 
 mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_budget budget,

@@ -64,6 +64,7 @@ __device__ __forceinline__ double ucb_value(u32 w, u32 k, u32 unit, double ln_pa
 struct LeafInfo {
   u64 own, opp;
   u32 term;
+  u32 refused;  // lane 0: the node wanted its first child but the pool was full (R12)
   int depth;
 };
 
@@ -103,6 +104,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
   }
   // Expansion (L179-L182): the lowest-index untried move, or the pass child.
   LeafInfo L;
+  L.refused = 0;
   if (!meta_term(meta)) {
     u32 c = kNoChild;
     if (lane == 0) {
@@ -115,6 +117,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
           T.first[base + v] = first;
         } else {
           first = kNoChild;  // pool full (time mode): simulate from v itself
+          L.refused = 1;
         }
       }
       if (first != kNoChild) {
@@ -162,7 +165,16 @@ __device__ __forceinline__ void backprop(const TreePool& T, size_t base, const u
 
 // Fused root merge (a10): add this tree's root-child statistics into the int64
 // stats vector (see MCTS_STATS_LEN in include/mcts.h). Integer atomics are
-// order-independent, so the sum is deterministic.
+// order-independent, so the sum is deterministic. Also the pool diagnostics:
+// [199] refused expansions, [200] slots used, [201] slot capacity.
+__device__ __forceinline__ void merge_pool(long long* stats, unsigned long long refused, u32 used,
+                                           u32 cap) {
+  unsigned long long* st = reinterpret_cast<unsigned long long*>(stats);
+  if (refused) atomicAdd(st + 199, refused);
+  atomicAdd(st + 200, (unsigned long long)used);
+  atomicAdd(st + 201, (unsigned long long)cap);
+}
+
 __device__ __forceinline__ void merge_root(const TreePool& T, size_t base, u32 unit, u32 iterations,
                                            long long* stats, int lane) {
   const u32 meta = T.meta[base];

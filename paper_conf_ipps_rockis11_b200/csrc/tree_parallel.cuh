@@ -115,9 +115,13 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
     path[0] = 0;
     atomicAdd(&T.vl[0], 1u);
   }
+  u32 refused = 0;
   for (;;) {
     if (meta_term(meta) || depth >= kMaxPath - 2) break;
-    if (first == kNoChild) break;  // pool full when v was created (or a racing read): simulate from v
+    if (first == kNoChild) {  // pool full when v was created (or a racing read): simulate from v
+      refused = 1;
+      break;
+    }
     // Expansion: claim the lowest-index untried move (one CAS on the counter).
     if (meta_nchild(meta) < meta_limit(meta)) {
       u32 claimed = kNoChild, mnow = meta;
@@ -195,6 +199,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
   L.own = __ldcg(&T.own[v]);
   L.opp = __ldcg(&T.opp[v]);
   L.term = meta_term(ld_acq(&T.meta[v])) ? 1u : 0u;
+  L.refused = refused;
   L.depth = depth;
   return L;
 }
@@ -236,6 +241,7 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
   u32 plies = 0;
   u32 done = 0;
   unsigned long long depth_sum = 0;  // lane 0 of warp 0
+  unsigned long long refused = 0;    // lane 0 of warp 0
   if (!meta_term(ld_acq(&T.meta[0]))) {
     for (;;) {
       if (warp == 0) {
@@ -254,6 +260,7 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth; s_it = it;
             depth_sum += (unsigned)L.depth;
+            refused += L.refused;
           }
         }
         if (lane == 0) s_stop = stop;
@@ -291,12 +298,31 @@ tree_search_kernel(TreePool T, SearchArgs a, TreeSync* S) {
     if (lane == 0 && P) atomicAdd(st + 197, P);
     if (lane == 0 && done) atomicAdd(st + 196, (unsigned long long)done);
     if (lane == 0 && depth_sum) atomicAdd(st + 198, depth_sum);
+    if (lane == 0 && refused) atomicAdd(st + 199, refused);
   }
 }
 
-// Root merge (a10) of the shared tree, after the search kernel (stream order).
-__global__ void tree_merge_kernel(TreePool T, u32 unit, long long* stats) {
+// Root merge (a10) of the shared tree, after the search kernel (stream order),
+// plus the pool diagnostics [200] slots used, [201] capacity (see merge_pool).
+__global__ void tree_merge_kernel(TreePool T, const TreeSync* S, u32 unit, long long* stats) {
   merge_root(T, 0, unit, 0u, stats, threadIdx.x & 31);
+  if (threadIdx.x == 0 && !meta_term(T.meta[0]))
+    merge_pool(stats, 0ULL, S->used < T.slot_cap ? S->used : T.slot_cap, T.slot_cap);
+}
+
+// Before a search: clear the fields a racing reader may see (meta = 0:
+// unpublished; k = w = vl = 0; first = kNoChild) over the slots the previous
+// search of this pool carving used (S->used, clamped to the capacity); the
+// rest of the pool is still clean from the last full clear.
+__global__ void tree_clear_kernel(TreePool T, const TreeSync* S) {
+  const u32 n = S->used < T.slot_cap ? S->used : T.slot_cap;
+  for (u32 s = blockIdx.x * blockDim.x + threadIdx.x; s < n; s += gridDim.x * blockDim.x) {
+    T.meta[s] = 0u;
+    T.k[s] = 0u;
+    T.w[s] = 0u;
+    T.vl[s] = 0u;
+    T.first[s] = kNoChild;
+  }
 }
 
 // Invariants of the finished tree (MCTS_FLAG_CHECK_TREE): every published node

@@ -2,7 +2,7 @@
 
 positions: int64 tensor [n, 3] (black, white, to_move | reserved << 32) = 24 B
 wdl:       int32 tensor [n, 3] (wins, draws, losses)
-stats:     int64 tensor [199]  (include/mcts.h MCTS_STATS_LEN)
+stats:     int64 tensor [202]  (include/mcts.h MCTS_STATS_LEN)
 """
 from __future__ import annotations
 

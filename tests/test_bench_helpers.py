@@ -125,3 +125,37 @@ def test_play_match_seed_base():
     got.clear()
     bench.play_match(mover("a"), 0, 2, 1.0, opp_move=mover("b"))
     assert max(got["a"]) < 100000
+
+
+def test_headline_plies_per_s_uses_the_kernel_time():
+    """plies_per_s and value divide by the same max-over-ranks device time
+    (round 1 divided plies by the shared-tree leg's 500 ms)."""
+    h = bench.headline(playouts_total=20 * 4096 * 256, plies_total=20 * 31_433_234, t_ms_max=20 * 0.3795,
+                       steps=20)
+    assert abs(h["plies_per_s"] - 31_433_234 / 0.3795e-3) < 1e-3 * h["plies_per_s"]
+    assert abs(h["value"] - 4096 * 256 / 0.3795e-3) < 1e-3 * h["value"]
+    assert h["ms_per_step"] == 0.3795 * 20 / 20
+    assert abs(h["plies_per_s"] / h["value"] - 31_433_234 / (4096 * 256)) < 1e-9
+
+
+def test_roofline_both_fractions():
+    r = bench.roofline(plies_per_launch=31_433_234, kern_s=0.3795e-3, peak_ops=3.572317e13, ops_exec=283.8,
+                       ops_basis="x", alu_peak=1.85e13, peak_basis="y")
+    assert abs(r["frac"] - 31_433_234 * bench.ALG_OPS_PER_PLY / 0.3795e-3 / 3.572317e13) < 1e-9
+    assert abs(r["frac_executed"] - 31_433_234 * 283.8 / 0.3795e-3 / 3.572317e13) < 1e-9
+    assert r["bound"] == "alu" and r["achieved"] == r["frac"] * r["peak"]
+
+
+def test_self_launch_cmd():
+    assert bench.self_launch_cmd(1, [], {}) is None
+    cmd = bench.self_launch_cmd(4, ["--gpus", "4", "--steps", "3"], {})
+    assert cmd[1:3] == ["-m", "torch.distributed.run"] and "--nproc-per-node=4" in cmd
+    assert "127.0.0.1" in cmd and cmd[-4:] == ["--gpus", "4", "--steps", "3"]
+    assert bench.self_launch_cmd(2, [], {"WORLD_SIZE": "2"}) is None
+    import pytest
+    with pytest.raises(SystemExit):
+        bench.self_launch_cmd(2, [], {"WORLD_SIZE": "4"})
+
+
+def test_kernel_source_hash_is_stable():
+    assert bench.kernel_source_hash() == bench.kernel_source_hash() and len(bench.kernel_source_hash()) == 16

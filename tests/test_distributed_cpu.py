@@ -34,7 +34,7 @@ def _worker(rank, world, port, q):
         root = oracle.gen_positions(21, 1, 20, 30)
         n = 5
         local, _, _ = oracle.uct_search(root, n, 32, 12, seed=4, tree_id_base=tree_id_base(rank, n))
-        st = torch.from_numpy(local.astype(np.int64))  # MCTS_STATS_LEN layout (199)
+        st = torch.from_numpy(local.astype(np.int64))  # MCTS_STATS_LEN layout (202)
         merge_root_stats(st)
         # leaf-range sharding of a playout batch (no collective on the data path)
         leaves = oracle.gen_positions(2, 11, 20, 40)
@@ -86,7 +86,7 @@ def test_leaf_range_partition():
 
 def test_merge_is_noop_single_process():
     from paper_conf_ipps_rockis11_b200.distributed import merge_root_stats, best_move_from
-    t = torch.arange(199, dtype=torch.int64)
+    t = torch.arange(202, dtype=torch.int64)
     assert torch.equal(merge_root_stats(t.clone()), t)
-    s = np.zeros(199, dtype=np.int64)
+    s = np.zeros(202, dtype=np.int64)
     assert best_move_from(s) == -1

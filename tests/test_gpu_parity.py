@@ -143,7 +143,7 @@ def test_playouts_leaf_range_sharding(mcts, orc):
 
 # ---------------------------------------------------------------- search
 def _cmp_search(res, ostats, obest):
-    assert res["stats"][:199].tolist() == ostats[:199].tolist()
+    assert res["stats"][:200].tolist() == ostats[:200].tolist()
     assert res["best_move"] == obest
 
 
@@ -196,7 +196,7 @@ def test_search_async_tree_id_base_merge_identity(mcts, orc):
     ostats, _, _ = orc.uct_search(root, n, 64, 15, 9, tree_id_base=2 * n)
     mcts.search_async(root, 15, 0.0, n, 64, 9, 2 * n, part.data_ptr(), torch.cuda.current_stream())
     torch.cuda.synchronize()
-    assert part.cpu().numpy()[:199].tolist() == ostats[:199].tolist()
+    assert part.cpu().numpy()[:200].tolist() == ostats[:200].tolist()
 
 
 def test_search_leaf_bit_exact(mcts_leaf, orc):
@@ -335,10 +335,10 @@ def test_search_hybrid_iteration_mode(mcts, orc):
     res = mcts.search_hybrid(root, iterations=40, n_trees=6, threads_per_tree=64, seed=12, cpu_threads=3)
     g, _, gp = orc.uct_search(root, 6, 64, 40, 12)
     c, _, cp = orc.uct_search(root, 3, 1, 40, 12, tree_id_base=0x40000000)
-    assert res["cpu"]["stats"][:199].tolist() == c[:199].tolist()
+    assert res["cpu"]["stats"][:200].tolist() == c[:200].tolist()
     assert res["cpu"]["plies"] == cp
     merged = g + c
-    assert res["stats"][:199].tolist() == merged[:199].tolist()
+    assert res["stats"][:200].tolist() == merged[:200].tolist()
     assert res["best_move"] == int(np.argmax(merged[:65]))
     assert res["plies"] == gp + cp
 
@@ -394,3 +394,47 @@ def test_device_perft_random_positions(mcts, orc):
         for depth in (3, 6):
             want = orc.perft(int(p["black"]), int(p["white"]), int(p["to_move"]), depth, True)
             assert mcts.perft(pos, depth, True) == want
+
+
+# ---------------------------------------------------------------- node-pool saturation (stats [199]-[201])
+def test_pool_counters_iteration_mode(mcts, orc):
+    root = orc.gen_positions(71, 1, 20, 30)
+    res = mcts.search(root, iterations=50, n_trees=4, threads_per_tree=64, seed=3)
+    s = res["stats"]
+    assert s[199] == 0 and res["refused_expansions"] == 0
+    assert 0 < s[200] <= s[201] and s[201] == 4 * (1 + 60 * 50)
+
+
+@pytest.mark.parametrize("scheme,n_trees,threads", [("block", 16, 64), ("tree", 64, 64), ("leaf", 1, 128)])
+def test_pool_full_is_counted(orc, scheme, n_trees, threads):
+    """A 64-slot pool fills within 20 ms: refused expansions are counted and
+    used slots never exceed the capacity."""
+    m = pkg.Mcts(c_uct=1.0, scheme=scheme, max_nodes_per_tree=64, device=0)
+    root = orc.gen_positions(17, 1, 20, 30)
+    res = m.search(root, time_ms=20.0, n_trees=n_trees, threads_per_tree=threads, seed=5)
+    s = res["stats"]
+    assert s[199] > 0
+    assert s[200] <= s[201] == (n_trees if scheme != "tree" else 1) * 64
+    assert s[195] == res["iterations"] * threads and s[:65].sum() == s[195]
+    m.close()
+
+
+def test_default_pool_does_not_saturate_in_500ms(mcts, orc):
+    """configs[2] at 500 ms from the opening with the default (time-sized) pool:
+    no expansion is refused."""
+    res = mcts.search(pkg.opening(), time_ms=500.0, n_trees=1184, threads_per_tree=128, seed=9)
+    s = res["stats"]
+    assert res["iterations"] > 1184 * 100
+    assert s[199] == 0, (s[199], s[200], s[201])
+    assert s[200] < s[201]
+
+
+def test_time_mode_rejects_non_resident_grid(mcts, orc):
+    """Time mode: trees that cannot be co-resident would start after the
+    deadline, so the call is rejected instead of silently running fewer trees."""
+    with pytest.raises(pkg.MctsError) as ei:
+        mcts.search(pkg.opening(), time_ms=10.0, n_trees=148 * 64, threads_per_tree=128, seed=1)
+    assert ei.value.status == -1
+    # iteration mode runs any grid (CTAs simply queue)
+    res = mcts.search(pkg.opening(), iterations=2, n_trees=148 * 20, threads_per_tree=32, seed=1)
+    assert res["iterations"] == 2 * 148 * 20

@@ -27,7 +27,7 @@ def test_tree_single_worker_config0_bit_exact(orc):
     m = _tree()
     res = m.search(pkg.opening(), iterations=100, n_trees=1, threads_per_tree=64, seed=1)
     ostats, obest, oplies = orc.uct_search(orc.opening(), 1, 64, 100, 1)
-    assert res["stats"][:199].tolist() == ostats[:199].tolist()
+    assert res["stats"][:200].tolist() == ostats[:200].tolist()
     assert res["best_move"] == obest and res["plies"] == oplies
     m.close()
 
@@ -44,7 +44,7 @@ def test_tree_single_worker_bit_exact(orc, threads, iters, seed, C, lmin, lmax):
     root = orc.gen_positions(seed, 1, lmin, lmax)
     res = m.search(root, iterations=iters, n_trees=1, threads_per_tree=threads, seed=seed)
     ostats, obest, oplies = orc.uct_search(root, 1, threads, iters, seed, C=C)
-    assert res["stats"][:199].tolist() == ostats[:199].tolist()
+    assert res["stats"][:200].tolist() == ostats[:200].tolist()
     assert res["best_move"] == obest and res["plies"] == oplies
     m.close()
 
@@ -57,7 +57,7 @@ def test_tree_single_worker_tree_id_base(orc):
     m.search_async(root, 40, 0.0, 1, 64, 3, 5, st.data_ptr(), torch.cuda.current_stream())
     torch.cuda.synchronize()
     ostats, _, _ = orc.uct_search(root, 1, 64, 40, 3, tree_id_base=5)
-    assert st.cpu().numpy()[:199].tolist() == ostats[:199].tolist()
+    assert st.cpu().numpy()[:200].tolist() == ostats[:200].tolist()
     m.close()
 
 
@@ -70,7 +70,7 @@ def test_tree_terminal_and_pass_roots(orc):
     root = orc.position(0b11, 0b100, 1)
     res = m.search(root, iterations=6, n_trees=1, threads_per_tree=32, seed=2)
     ostats, obest, _ = orc.uct_search(root, 1, 32, 6, 2)
-    assert res["stats"][:199].tolist() == ostats[:199].tolist() and res["best_move"] == 64
+    assert res["stats"][:200].tolist() == ostats[:200].tolist() and res["best_move"] == 64
     m.close()
 
 
@@ -140,7 +140,7 @@ def test_tree_hybrid_iteration_mode(orc):
     g, _, gp = orc.uct_search(root, 1, 64, 60, 14)
     c, _, cp = orc.uct_search(root, 3, 1, 60, 14, tree_id_base=0x40000000)
     merged = g + c
-    assert res["stats"][:199].tolist() == merged[:199].tolist()
+    assert res["stats"][:200].tolist() == merged[:200].tolist()
     assert res["plies"] == gp + cp
     m.close()
 

@@ -189,11 +189,11 @@ def test_mcts_timed_capped_equals_uct_search(orc, threads, iters, seed, C, lmin,
     """The root-parallel CPU opponent, capped at `iters`
     iterations per thread with no deadline, is T independent unit-1 trees keyed
     (c0 = thread, c1 = iteration, c2 = 0) summed at the root: bit for bit
-    uct_search(root, T, 1, iters, seed) — all 199 stats and the move."""
+    uct_search(root, T, 1, iters, seed) — the root stats, counters and the move."""
     root = orc.gen_positions(seed, 1, lmin, lmax) if lmax else orc.opening()
     got, best = orc.mcts_timed(root, threads, 0.0, seed, C=C, max_iterations=iters)
     want, wbest, plies = orc.uct_search(root, threads, 1, iters, seed, C=C)
-    assert got.tolist() == want.tolist()
+    assert got[:201].tolist() == want[:201].tolist()  # [201]: the opponent's pool is unbounded
     assert best == wbest
     assert got[196] == threads * iters and got[195] == threads * iters and got[197] == plies
 
@@ -203,7 +203,7 @@ def test_mcts_timed_cap_with_generous_deadline(orc):
     root = orc.gen_positions(11, 1, 20, 30)
     got, best = orc.mcts_timed(root, 2, 60000.0, 4, C=0.5, max_iterations=100)
     want, wbest, _ = orc.uct_search(root, 2, 1, 100, 4, C=0.5)
-    assert got.tolist() == want.tolist() and best == wbest
+    assert got[:201].tolist() == want[:201].tolist() and best == wbest
 
 
 def test_mcts_timed_time_mode_invariants(orc):
@@ -223,3 +223,25 @@ def test_mcts_timed_terminal_root(orc):
     s, best = orc.mcts_timed(orc.position(full_black, ((1 << 64) - 1) & ~full_black, 0), 2, 0.0, 1,
                              max_iterations=10)
     assert best == -1 and (s == 0).all()
+
+
+@pytest.mark.parametrize("seed,cap,lmin,lmax", [(5, 40, 20, 30), (6, 12, 40, 50), (7, 300, 0, 10)])
+def test_refused_expansions_counter(orc, seed, cap, lmin, lmax):
+    """stats[199] (expansions refused by a full pool, R12) from the tree dump:
+    every iteration either expands one node, ends at a terminal node, or is
+    refused, so refused = iterations - (nodes - 1) - sum over terminal nodes
+    of (visits / unit - 1) (the iteration that created a terminal node ended
+    there as its expansion). [200] = nodes, [201] = capacity."""
+    unit, iters = 32, 400
+    root = orc.gen_positions(seed, 1, lmin, lmax)
+    s, _, _ = orc.uct_search(root, 1, unit, iters, seed, capacity=cap)
+    t = orc.uct_tree(root, unit, iters, seed, tree_id=0, C=1.0, capacity=cap)
+    nodes = len(t["parent"])
+    term_ends = sum(int(n) // unit - 1 for n, term, par in zip(t["n"], t["terminal"], t["parent"])
+                    if term and par >= 0)
+    assert s[199] == iters - (nodes - 1) - term_ends
+    assert s[200] == nodes and s[201] == cap
+    if nodes == cap:
+        assert s[199] > 0
+    s0, _, _ = orc.uct_search(root, 1, unit, iters, seed)  # iteration-mode pool: never refuses
+    assert s0[199] == 0 and s0[:199].tolist() != [] and s0[201] == iters + 1

@@ -5,6 +5,8 @@ sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from ncu_summary import summary
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench  # noqa: E402  (kernel_source_hash: the sources this capture was built from)
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 out_dir = os.path.join(ROOT, "profiles")
 os.makedirs(out_dir, exist_ok=True)
@@ -42,7 +44,8 @@ for k in ["playouts", "block_search", "leaf_search", "tree_search"]:
                  "dram_bytes_per_launch": num("dram__bytes_read.sum") + num("dram__bytes_write.sum"),
                  "duration_us": num("gpu__time_duration.sum"),
                  "thread_inst": float(d["smsp__inst_executed.sum"][0].replace(",", "")) *
-                 float(d["smsp__thread_inst_executed_per_inst_executed.ratio"][0])}
+                 float(d["smsp__thread_inst_executed_per_inst_executed.ratio"][0]),
+                 "source_hash": bench.kernel_source_hash(), "capture": f"profiles/{tag}_ncu_{k}.txt"}
     if k == "playouts":  # the captured launch is one configs[1] batch (bench.py default workload)
         try:
             b = json.loads(open(os.path.join(ROOT, "gpurun_out", f"{tag}_bench.json")).read().splitlines()[-1])
