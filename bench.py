@@ -241,7 +241,12 @@ def sweep_leg(args, local):
                 continue
             n_trees, threads = (1, total) if scheme == "leaf" else (total // bs, bs)
             h = handles[scheme]
-            h.search_async(root, 0, 10.0, n_trees, threads, 7, 0, st.data_ptr(), stream)  # warm-up
+            try:
+                h.search_async(root, 0, 10.0, n_trees, threads, 7, 0, st.data_ptr(), stream)  # warm-up
+            except pkg.MctsError as e:  # time mode needs every tree co-resident (trees beyond would idle)
+                points.append({"scheme": scheme, "block": bs, "gpu_threads": total, "trees": n_trees,
+                               "skipped": str(e)})
+                continue
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
