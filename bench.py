@@ -56,7 +56,7 @@ def kernel_source_hash() -> str:
     import hashlib
     from paper_conf_ipps_rockis11_b200 import _build
     h = hashlib.sha256()
-    for name in ("reversi_device.cuh", "kernels.cuh"):
+    for name in ("reversi_device.cuh", "playouts.cuh"):
         h.update(open(os.path.join(_build.CSRC, name), "rb").read())
     h.update(" ".join(_build.NVCC_FLAGS).encode())
     return h.hexdigest()[:16]
@@ -700,8 +700,9 @@ def main():
         root = pkg.position(*pkg.OPENING)
         st = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
         it, ms = (args.search_iters * it_scale, 0.0) if args.search_iters else (0, args.search_ms)
-        handle.search_async(root, min(it, 2) if it else 0, 0.0 if it else 20.0, n_trees, threads,
-                            1000, id_base, st.data_ptr(), stream)  # warm-up: pool + ln table
+        # warm-up with the same budget: the time-sized node pool and the ln table
+        # are allocated here, not inside the timed search
+        handle.search_async(root, it, ms, n_trees, threads, 999, id_base, st.data_ptr(), stream)
         torch.cuda.synchronize()
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

@@ -11,95 +11,17 @@
 //   gen_positions_kernel synthetic input recipe
 #pragma once
 #include <cstdint>
-#include <cooperative_groups.h>
 #include "reversi_device.cuh"
 #include "ln_device.cuh"
 #include "tree_device.cuh"
+#include "playouts.cuh"
 
 namespace mcts_dev {
-
-struct DevPosition {  // layout of mcts_position
-  u64 black, white;
-  u32 to_move, reserved;
-};
-
-struct WdlOut {  // layout of mcts_wdl
-  u32 wins, draws, losses;
-};
 
 __device__ __forceinline__ u64 globaltimer_ns() {
   u64 t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
-}
-
-// ---------------------------------------------------------------------------
-// Batched playouts, persistent: the grid is sized to the resident capacity and
-// each warp repeatedly takes the next chunk of 32 playouts from a work counter
-// (dynamic balancing; the per-CTA ray table is loaded once). Playout g of a
-// launch is playout j = g mod n_per_leaf of leaf g / n_per_leaf (leaf-major, so
-// a warp's 32 lanes usually share a leaf and finish within a ply or two of each
-// other). Outcomes are reduced per (warp, leaf) with match_any + ballot + popc
-// and added with one atomic per counter; plies with one atomic per warp.
-// ---------------------------------------------------------------------------
-#ifndef MCTS_PLAYOUT_THREADS
-#define MCTS_PLAYOUT_THREADS 256
-#endif
-#ifndef MCTS_PLAYOUT_MINB
-#define MCTS_PLAYOUT_MINB 1
-#endif
-constexpr int kPlayoutThreads = MCTS_PLAYOUT_THREADS;
-
-__global__ void rays_init_kernel(u64* g_rays) {
-  fill_rays(g_rays);
-}
-
-__device__ __forceinline__ void load_rays(u64* s_rays, const u64* __restrict__ g_rays) {
-  for (int i = threadIdx.x; i < kRayTable; i += blockDim.x) s_rays[i] = g_rays[i];
-}
-
-__global__ void __launch_bounds__(kPlayoutThreads, MCTS_PLAYOUT_MINB)
-playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
-                u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out,
-                const u64* __restrict__ g_rays, u32* __restrict__ work) {
-  __shared__ u64 s_rays[kRayTable];
-  load_rays(s_rays, g_rays);
-  __syncthreads();
-  const u64 total = (u64)n_leaves * n_per_leaf;
-  const u32 n_chunks = (u32)((total + 31) / 32);
-  const int lane = threadIdx.x & 31;
-  u32 plies = 0;
-  for (;;) {
-    u32 chunk = 0;
-    if (lane == 0) chunk = atomicAdd(work, 1u);
-    chunk = __shfl_sync(kFull, chunk, 0);
-    if (chunk >= n_chunks) break;
-    const u64 g = (u64)chunk * 32u + (u32)lane;
-    const bool active = g < total;
-    u32 leaf = 0xFFFFFFFFu;
-    int r = 2;
-    if (active) {
-      leaf = (u32)(g / n_per_leaf);
-      const u32 j = (u32)(g - (u64)leaf * n_per_leaf);
-      const DevPosition p = leaves[leaf];
-      const u64 own = p.to_move ? p.white : p.black;
-      const u64 opp = p.to_move ? p.black : p.white;
-      r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, s_rays, &plies);
-    }
-    const u32 grp = __match_any_sync(kFull, leaf);
-    const u32 wins = __popc(__ballot_sync(kFull, r == 1) & grp);
-    const u32 draws = __popc(__ballot_sync(kFull, r == 0) & grp);
-    const u32 losses = __popc(__ballot_sync(kFull, r == -1) & grp);
-    if (active && lane == __ffs(grp) - 1) {
-      if (wins) atomicAdd(&out[leaf].wins, wins);
-      if (draws) atomicAdd(&out[leaf].draws, draws);
-      if (losses) atomicAdd(&out[leaf].losses, losses);
-    }
-  }
-  if (plies_out) {
-    const u32 s = __reduce_add_sync(kFull, plies);
-    if (lane == 0 && s) atomicAdd(plies_out, (unsigned long long)s);
-  }
 }
 
 // ---------------------------------------------------------------------------
@@ -213,22 +135,68 @@ block_search_kernel(TreePool T, SearchArgs a) {
 
 // ---------------------------------------------------------------------------
 // Leaf-parallel UCT: one tree; every thread of the grid
-// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree
-// (select/expand/backprop); the leaf is published through a small global
-// struct between two cooperative-groups grid barriers per iteration
-// (select -> sync -> simulate + per-CTA ballot reduce + atomics -> sync).
-// All CTAs are co-resident (cooperative launch).
+// plays out from the same leaf each iteration. CTA 0's warp 0 (the leader)
+// owns the tree (select/expand/backprop); all CTAs are co-resident
+// (cooperative launch). One grid-wide hand-off per iteration instead of two
+// barriers:
+//   leader: publishes the iteration's leaf in S, then gen = it + 1 (release);
+//   every CTA: waits for gen > it (acquire), plays its playouts, reduces them
+//     (ballots + shared memory), adds (W, D) to S->wd[it & 1] and then bumps
+//     S->done[it & 1] (fence + atomic: release);
+//   leader: waits for done[it & 1] == gridDim (acquire), takes and clears the
+//     sums, backpropagates, selects the next leaf and publishes it.
+// The parity double-buffer makes the clears safe: slot it & 1 is next written
+// in iteration it + 2, which no CTA reaches before the leader publishes it.
+// Only the leader touches the tree, so its reads never see another SM's stale
+// L1 lines; the hand-off words are read with L2 (.cg / acquire) loads.
 // ---------------------------------------------------------------------------
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
+  u32 gen;          // iterations whose leaf has been published
+  u32 done[2];      // CTAs finished with iteration it (parity it & 1)
   u32 wd[2][2];     // per-iteration-parity wins, draws
 };
 
+__device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u32(u32* p, u32 v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// The leader warp selects iteration `it`'s leaf (or decides to stop) and
+// publishes it: S fields, then gen = it + 1 with release semantics.
+__device__ __forceinline__ void leaf_select_publish(const TreePool& T, const SearchArgs& a, LeafSync* S,
+                                                    u32* path, u32* slot_used, int* s_depth, u32 it,
+                                                    u64 deadline, int lane, unsigned long long& depth_sum,
+                                                    unsigned long long& refused) {
+  u32 stop = 0;
+  if (lane == 0) {
+    stop = meta_term(T.meta[0]) || it >= a.max_iterations;
+    if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
+  }
+  stop = __shfl_sync(kFull, stop, 0);
+  if (!stop) {
+    const LeafInfo L = select_expand(T, 0, path, slot_used, a.lnT, a.unit, a.C, lane);
+    if (lane == 0) {
+      *s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
+      depth_sum += (unsigned)L.depth;
+      refused += L.refused;
+    }
+  }
+  if (lane == 0) {
+    S->stop = stop;
+    __threadfence();
+    st_release_u32(&S->gen, it + 1u);
+  }
+  __syncwarp();
+}
+
 __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
-  namespace cg = cooperative_groups;
-  cg::grid_group grid = cg::this_grid();
   __shared__ u32 path[kMaxPath];
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
@@ -239,48 +207,40 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const bool leader = blockIdx.x == 0 && warp == 0;
   const u32 unit = a.unit;
+  const u32 G = gridDim.x;
   const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
-  if (blockIdx.x == 0 && tid == 0) {
+  u32 plies = 0;
+  unsigned long long depth_sum = 0;  // leader lane 0
+  unsigned long long refused = 0;    // leader lane 0
+
+  if (leader && lane == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
     const u64 opp = a.root.to_move ? a.root.black : a.root.white;
     init_node(T, 0, own, opp, 0xFFu);
     s_slot_used = 1;
   }
-  __syncthreads();
-  u32 plies = 0;
   u32 it = 0;
-  unsigned long long depth_sum = 0;  // leader lane 0
-  unsigned long long refused = 0;    // leader lane 0
   for (;; ++it) {
     if (leader) {
-      if (it > 0) {
-        const u32 par = (it - 1) & 1u;
-        const u32 W = S->wd[par][0], D = S->wd[par][1];
+      if (it > 0) {  // collect iteration it - 1 from every CTA, backpropagate
+        const u32 pp = (it - 1u) & 1u;
+        if (lane == 0)
+          while (ld_acquire_u32(&S->done[pp]) < G) __nanosleep(20);
         __syncwarp();
-        if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
+        const u32 W = __ldcg(&S->wd[pp][0]), D = __ldcg(&S->wd[pp][1]);
+        __syncwarp();
+        if (lane == 0) { S->wd[pp][0] = 0; S->wd[pp][1] = 0; S->done[pp] = 0; }
         backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
       }
-      u32 stop = 0;
-      if (lane == 0) {
-        stop = meta_term(T.meta[0]) || it >= a.max_iterations;
-        if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
-      }
-      stop = __shfl_sync(kFull, stop, 0);
-      if (!stop) {
-        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
-        if (lane == 0) {
-          s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
-          depth_sum += (unsigned)L.depth;
-          refused += L.refused;
-        }
-      }
-      if (lane == 0) S->stop = stop;
+      leaf_select_publish(T, a, S, path, &s_slot_used, &s_depth, it, deadline, lane, depth_sum, refused);
     }
-    grid.sync();
-    const u32 stop = S->stop;
-    const u64 own = S->own, opp = S->opp;
-    const u32 term = S->term;
+    if (tid == 0)
+      while (ld_acquire_u32(&S->gen) <= it) __nanosleep(32);
+    __syncthreads();
+    const u32 stop = __ldcg(&S->stop);
     if (stop) break;
+    const u64 own = __ldcg(&S->own), opp = __ldcg(&S->opp);
+    const u32 term = __ldcg(&S->term);
     int r;
     if (term) {
       const int x = __popcll(own), y = __popcll(opp);
@@ -296,8 +256,9 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       const u32 par = it & 1u;
       atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
       atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
+      __threadfence();
+      atomicAdd(&S->done[par], 1u);
     }
-    grid.sync();
   }
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
