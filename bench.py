@@ -289,6 +289,7 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
     res = {"W": 0, "D": 0, "L": 0}
     diffs, gpu_po, cpu_po, steps = [], [], [], []
     depth = {"gpu": {}, "opp": {}}  # game step -> mean tree depths (searchers that report one)
+    pool = {"refused": 0, "max_fill": 0.0}  # node-pool saturation of the GPU searcher over all moves
     t_start = time.time()
     for g in range(games):
         gpu_color = g % 2
@@ -308,6 +309,9 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
                 gpu_po.append(po)
                 if dp:
                     depth["gpu"].setdefault(ply, []).append(dp[0])
+                if len(dp) > 1:  # (refused expansions, slots used, slot capacity) of this move's search
+                    pool["refused"] += dp[1][0]
+                    pool["max_fill"] = max(pool["max_fill"], dp[1][1] / max(dp[1][2], 1))
             elif opp_move is not None:  # another device searcher (--h2h)
                 mv, po, *dp = opp_move(black, white, to_move, seed + 500)
                 cpu_po.append(po)
@@ -345,6 +349,7 @@ def play_match(gpu_move, cpu_threads, games, move_ms, seed_base=1000, tag="", op
             # mean depth of the simulated node per game step (the paper's Fig. 8 "Depth")
             "gpu_depth_per_step": {int(k): float(np.mean(v)) for k, v in sorted(depth["gpu"].items())},
             "opp_depth_per_step": {int(k): float(np.mean(v)) for k, v in sorted(depth["opp"].items())},
+            "gpu_refused_expansions": pool["refused"], "gpu_pool_max_fill": pool["max_fill"],
             "wall_s": time.time() - t_start}
 
 
@@ -370,7 +375,8 @@ def h2h_leg(args, local):
                            st.data_ptr(), stream)
             torch.cuda.synchronize()
             x = st.cpu().numpy()
-            return pkg.best_move(x), int(x[195]), float(x[198]) / max(int(x[196]), 1)
+            return (pkg.best_move(x), int(x[195]), float(x[198]) / max(int(x[196]), 1),
+                    (int(x[199]), int(x[200]), int(x[201])))
         return move
 
     r = play_match(mover(ha, *SCHEME_SHAPE[a]), 0, args.selfplay, args.move_ms, tag="h2h",
@@ -420,14 +426,16 @@ def selfplay_leg(args, world, rank, local):
         if hybrid:  # NEXT-1: GPU trees + one host tree per host core, root sums merged
             r = m.search_hybrid(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads,
                                 seed=seed, cpu_threads=len(os.sched_getaffinity(0)))
-            return r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1)
+            return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1),
+                    (r["refused_expansions"], r["slots_used"], r["slot_capacity"]))
         m.search_async(pos, 0, args.move_ms, n_trees, threads, seed, rank * n_trees,
                        stats.data_ptr(), stream)
         with torch.cuda.stream(stream):
             merge_root_stats(stats)
         torch.cuda.synchronize()
         st = stats.cpu().numpy()
-        return pkg.best_move(st), int(st[195]), float(st[198]) / max(int(st[196]), 1)
+        return (pkg.best_move(st), int(st[195]), float(st[198]) / max(int(st[196]), 1),
+                (int(st[199]), int(st[200]), int(st[201])))
 
     if rank != 0:  # follower ranks: search whatever position rank 0 broadcasts
         while True:

@@ -67,6 +67,8 @@ def lib() -> ctypes.CDLL:
         L.orc_uct_tree.restype = ctypes.c_int64
         L.orc_gen_positions.argtypes = [u64, u32, u32, u32, vp]; L.orc_gen_positions.restype = None
         L.orc_mcts_timed.argtypes = [vp, i32, dbl, u64, dbl, vp, u64]; L.orc_mcts_timed.restype = i32
+        L.orc_hybrid_search.argtypes = [vp, u32, u32, u64, u32, u64, u32, dbl, vp, vp, i32]
+        L.orc_hybrid_search.restype = i32
         _lib = L
     return _lib
 
@@ -190,3 +192,17 @@ def mcts_timed(root: np.ndarray, nthreads: int, budget_ms: float, seed: int, C: 
     stats = np.zeros(N_STATS, dtype=np.int64)
     best = lib().orc_mcts_timed(_ptr(root), nthreads, budget_ms, seed, C, _ptr(stats), max_iterations)
     return stats, int(best)
+
+
+def hybrid_search(root: np.ndarray, n_trees: int, unit: int, steps: int, cpu_iters: int, seed: int,
+                  tree_id_base: int = 0, C: float = 1.0, nthreads: int = 0):
+    """Hybrid CPU-GPU processing on CPU-managed trees (PAPER.md L312-L339, Fig. 4;
+    DESIGN.md R18): per step a GPU leaf of `unit` playouts, cpu_iters one-playout
+    CPU iterations on the same tree meanwhile, then the GPU backprop. Returns
+    (stats[202], best, cpu) with cpu = dict(iterations, plies, depth_sum, cpu_nodes, gpu_nodes)."""
+    stats = np.zeros(N_STATS, dtype=np.int64)
+    cpu = np.zeros(5, dtype=np.int64)
+    best = lib().orc_hybrid_search(_ptr(root), n_trees, unit, steps, cpu_iters, seed, tree_id_base, C,
+                                   _ptr(stats), _ptr(cpu), nthreads)
+    return stats, int(best), dict(iterations=int(cpu[0]), plies=int(cpu[1]), depth_sum=int(cpu[2]),
+                                  cpu_nodes=int(cpu[3]), gpu_nodes=int(cpu[4]))

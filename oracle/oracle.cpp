@@ -341,6 +341,143 @@ void search_tree(uint64_t root_own, uint64_t root_opp, uint32_t unit, uint64_t i
   if (plies_total) *plies_total += plies;
 }
 
+// ---------------------------------------------------------------------------
+// Hybrid CPU-GPU processing on CPU-managed trees (§III-A,
+// Fig. 4), on the block-parallel trees as the paper built them: "The trees are
+// still controlled by the CPU threads, GPU simulates only" (L302-L303). DESIGN.md
+// reading R18. Per tree, per step s:
+//   1. select + expand one leaf (the GPU's leaf of this step);
+//   2. GPU: `unit` playouts from it, streams (c0 = tree_id, c1 = s, c2 = 0..unit-1)
+//      — the block search's iteration-s streams;
+//   3. "CPU can work here!" (Fig. 4): cpu_iters UCT iterations on the SAME tree,
+//      one playout each, streams (c0 = tree_id, c1 = 0x80000000 + s*cpu_iters + j, c2 = 0);
+//   4. backpropagate step 2's result along step 1's path.
+// Selection is R1 with the parent's simulation count N (GPU steps add `unit`,
+// CPU iterations 1, so ln is RN(ln N) of any N) and one more rule: a child
+// with n = 0 — a leaf whose GPU simulations are still pending — is unvisited,
+// scored +inf as in UCB1 (ref [2]), lowest index first.
+// ---------------------------------------------------------------------------
+struct HybridCounts {
+  uint64_t cpu_iterations = 0, cpu_plies = 0, cpu_depth_sum = 0, cpu_nodes = 0, gpu_nodes = 0;
+};
+
+double ln_of(std::vector<double>& lnT, uint64_t N) {
+  if (N >= lnT.size()) {
+    size_t old = lnT.size();
+    lnT.resize(std::max<size_t>(N + 1, old * 2));
+    for (size_t k = old; k < lnT.size(); ++k) lnT[k] = ln_rn(k);
+  }
+  return lnT[N];
+}
+
+// Steps 1 (and the CPU iterations' selection + expansion): returns the path
+// root..leaf; *expanded = 1 if a node was added.
+std::vector<int> select_expand_pending(std::vector<Node>& nodes, double C, std::vector<double>& lnT,
+                                       int* expanded) {
+  std::vector<int> path;
+  int v = 0;
+  path.push_back(v);
+  while (!nodes[v].terminal && fully_expanded(nodes[v])) {
+    const Node& p = nodes[v];
+    int best = -1;
+    double best_u = -INFINITY;
+    for (int c : p.children) {
+      if (nodes[c].n == 0) { best = c; break; }  // pending: unvisited, +inf (first in index order)
+      double u = ucb(nodes[c].w, nodes[c].n, ln_of(lnT, p.n), C);
+      if (u > best_u) { best_u = u; best = c; }
+    }
+    v = best;
+    path.push_back(v);
+  }
+  *expanded = 0;
+  if (!nodes[v].terminal) {
+    const Node& p = nodes[v];
+    int mv;
+    uint64_t cown, copp;
+    if (p.legal_moves == 0) {
+      mv = 64;
+      cown = p.opp; copp = p.own;
+    } else {
+      int idx = (int)p.children.size(), seen = 0;
+      mv = -1;
+      for (int sq = 0; sq < 64; ++sq)
+        if ((p.legal_moves >> sq) & 1) { if (seen == idx) { mv = sq; break; } ++seen; }
+      uint64_t f = flips(p.own, p.opp, mv);
+      cown = p.opp & ~f; copp = p.own | f | (1ULL << mv);
+    }
+    nodes.push_back(make_node(cown, copp, mv, v));
+    int c = (int)nodes.size() - 1;
+    nodes[v].children.push_back(c);
+    path.push_back(c);
+    *expanded = 1;
+  }
+  return path;
+}
+
+// Results (wins, draws, losses for the leaf's side to move) of `count`
+// playouts from the leaf with streams (c0, c1, c2 = 0..count-1).
+void simulate(const Node& leaf, uint32_t count, uint64_t seed, uint32_t c0, uint32_t c1, uint64_t* wdl,
+              uint64_t* plies) {
+  wdl[0] = wdl[1] = wdl[2] = 0;
+  if (leaf.terminal) {
+    int a = popcount64(leaf.own), b = popcount64(leaf.opp);
+    wdl[a > b ? 0 : (a == b ? 1 : 2)] = count;
+    return;
+  }
+  for (uint32_t t = 0; t < count; ++t) {
+    uint32_t pl = 0;
+    int r = playout(leaf.own, leaf.opp, seed, c0, c1, t, &pl);
+    *plies += pl;
+    ++wdl[r > 0 ? 0 : (r == 0 ? 1 : 2)];
+  }
+}
+
+// Step 4 / the CPU iterations' backpropagation (L196-L199): n += count along
+// the path, w += wins of each node's mover, d += draws.
+void backprop_path(std::vector<Node>& nodes, const std::vector<int>& path, uint32_t count, const uint64_t* wdl) {
+  uint64_t mover_wins = wdl[2], other_wins = wdl[0];
+  for (int i = (int)path.size() - 1; i >= 0; --i) {
+    Node& x = nodes[path[i]];
+    x.n += count;
+    x.w += mover_wins;
+    x.d += wdl[1];
+    std::swap(mover_wins, other_wins);
+  }
+}
+
+void hybrid_tree(uint64_t root_own, uint64_t root_opp, uint32_t unit, uint64_t steps, uint32_t cpu_iters,
+                 uint64_t seed, uint32_t tree_id, double C, TreeResult* out, uint64_t* plies,
+                 HybridCounts* hc) {
+  std::vector<Node>& nodes = out->nodes;
+  nodes.clear();
+  nodes.push_back(make_node(root_own, root_opp, -1, -1));
+  out->iterations = 0;
+  if (nodes[0].terminal) return;
+  std::vector<double> lnT(1, 0.0);
+  for (uint64_t s = 0; s < steps; ++s) {
+    int e = 0;
+    std::vector<int> gpath = select_expand_pending(nodes, C, lnT, &e);  // 1
+    hc->gpu_nodes += e;
+    uint64_t g[3];
+    simulate(nodes[gpath.back()], unit, seed, tree_id, (uint32_t)s, g, plies);  // 2
+    out->depth_sum += gpath.size() - 1;
+    for (uint32_t j = 0; j < cpu_iters; ++j) {  // 3: on the same tree while the GPU works
+      std::vector<int> cpath = select_expand_pending(nodes, C, lnT, &e);
+      hc->cpu_nodes += e;
+      uint64_t c[3], cp = 0;
+      simulate(nodes[cpath.back()], 1, seed, tree_id, 0x80000000u + (uint32_t)(s * cpu_iters + j), c, &cp);
+      backprop_path(nodes, cpath, 1, c);
+      *plies += cp;
+      hc->cpu_plies += cp;
+      hc->cpu_iterations += 1;
+      hc->cpu_depth_sum += cpath.size() - 1;
+      out->depth_sum += cpath.size() - 1;
+    }
+    backprop_path(nodes, gpath, unit, g);  // 4
+    out->iterations += 1 + cpu_iters;
+  }
+}
+
 uint64_t perft_rec(uint64_t own, uint64_t opp, int depth, bool pass_is_ply) {
   if (depth == 0) return 1;
   uint64_t m = legal(own, opp);
@@ -568,6 +705,65 @@ void orc_gen_positions(uint64_t seed, uint32_t n, uint32_t lmin, uint32_t lmax, 
       break;
     }
   }
+}
+
+// Hybrid CPU-GPU search on CPU-managed trees (hybrid_tree above; the
+// mcts_search_hosted contract): n_trees trees (ids tree_id_base + t), `steps`
+// GPU steps of `unit` playouts each with cpu_iters CPU iterations per step.
+// stats as orc_uct_search ([196] counts GPU steps and CPU iterations, [197]
+// all plies, [198] both depth sums; [199] 0, [200] nodes, [201] 0 = unbounded);
+// cpu[0..4] = CPU iterations, CPU plies, CPU depth sum, nodes added by CPU
+// iterations, nodes added by GPU steps. cpu_iters = 0 is the block-parallel
+// search (uct_search) bit for bit. Returns the best move (R8).
+int orc_hybrid_search(const orc_position* root, uint32_t n_trees, uint32_t unit, uint64_t steps,
+                      uint32_t cpu_iters, uint64_t seed, uint32_t tree_id_base, double C, int64_t* stats,
+                      int64_t* cpu, int nthreads) {
+  for (int i = 0; i < 202; ++i) stats[i] = 0;
+  for (int i = 0; i < 5; ++i) cpu[i] = 0;
+  uint64_t own, opp;
+  to_own_opp(*root, &own, &opp);
+  std::vector<TreeResult> res(n_trees);
+  std::vector<uint64_t> plies(n_trees, 0);
+  std::vector<HybridCounts> hc(n_trees);
+  int T = std::min<int>(resolve_threads(nthreads), (int)std::max<uint32_t>(n_trees, 1));
+  std::atomic<uint32_t> next{0};
+  auto worker = [&]() {
+    for (;;) {
+      uint32_t t = next.fetch_add(1);
+      if (t >= n_trees) break;
+      hybrid_tree(own, opp, unit, steps, cpu_iters, seed, tree_id_base + t, C, &res[t], &plies[t], &hc[t]);
+    }
+  };
+  std::vector<std::thread> pool;
+  for (int t = 1; t < T; ++t) pool.emplace_back(worker);
+  worker();
+  for (auto& th : pool) th.join();
+  for (uint32_t t = 0; t < n_trees; ++t) {
+    const std::vector<Node>& nodes = res[t].nodes;
+    if (nodes[0].terminal) continue;
+    for (int c : nodes[0].children) {
+      int mv = nodes[c].move;
+      stats[mv] += (int64_t)nodes[c].n;
+      stats[65 + mv] += (int64_t)nodes[c].w;
+      stats[130 + mv] += (int64_t)nodes[c].d;
+    }
+    stats[195] += (int64_t)nodes[0].n;
+    stats[196] += (int64_t)res[t].iterations;
+    stats[197] += (int64_t)plies[t];
+    stats[198] += (int64_t)res[t].depth_sum;
+    stats[200] += (int64_t)nodes.size();
+    cpu[0] += (int64_t)hc[t].cpu_iterations;
+    cpu[1] += (int64_t)hc[t].cpu_plies;
+    cpu[2] += (int64_t)hc[t].cpu_depth_sum;
+    cpu[3] += (int64_t)hc[t].cpu_nodes;
+    cpu[4] += (int64_t)hc[t].gpu_nodes;
+  }
+  if (n_trees == 0 || res[0].nodes[0].terminal) return -1;
+  int best = -1;
+  int64_t bv = 0;
+  for (int mv = 0; mv < 65; ++mv)
+    if (stats[mv] > bv) { bv = stats[mv]; best = mv; }
+  return best;
 }
 
 // Root-parallel CPU MCTS opponent: one tree

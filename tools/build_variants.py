@@ -25,6 +25,11 @@ VARIANTS = {
     "zt0": ["MCTS_ZT=0"],
     "hxp0": ["MCTS_HXP=0"],
     "old3": ["MCTS_NW=0", "MCTS_ZT=0", "MCTS_HXP=0"],
+    "minb5": ["MCTS_PLAYOUT_MINB=5"],
+    "t128m9": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=9"],
+    "t128m10": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=10"],
+    "t128m11": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=11"],
+    "t64m20": ["MCTS_PLAYOUT_THREADS=64", "MCTS_PLAYOUT_MINB=20"],
 }
 
 if __name__ == "__main__":
