@@ -166,6 +166,14 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
                                 uint32_t n_per_leaf, uint64_t seed, uint32_t leaf_id_base,
                                 mcts_wdl* d_out, uint64_t* d_plies, void* stream);
 
+/* The same kernel with the full stream key: leaf i's playouts use (c0 =
+ * c0_base + i, c1, c2 = j). mcts_playouts_async is c1 = 0. This is the
+ * "GPU simulates only" half of the paper's CPU-managed trees (L302-L303):
+ * c1 = the step, so a step's batch reproduces the block search's iteration. */
+mcts_status mcts_playouts_ex_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
+                                   uint32_t n_per_leaf, uint64_t seed, uint32_t c0_base, uint32_t c1,
+                                   mcts_wdl* d_out, uint64_t* d_plies, void* stream);
+
 /* UCT search with the handle's scheme:
  *   MCTS_BLOCK: n_trees independent trees, one per CTA of threads_per_tree
  *               threads (multiple of 32, 32..1024); threads_per_tree playouts
@@ -212,6 +220,46 @@ mcts_status mcts_search_async(mcts_handle* h, const mcts_position* root, mcts_bu
 mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_budget budget,
                                uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
                                uint32_t cpu_threads, mcts_root_stats* out, mcts_root_stats* out_cpu);
+
+/* mcts_search_hosted diagnostics: how the work split between CPU and GPU. */
+typedef struct {
+  uint64_t steps;          /* GPU steps (one playout kernel over every tree's leaf) */
+  uint64_t cpu_iterations; /* UCT iterations the host threads ran on the same trees */
+  uint64_t cpu_plies;      /* plies of their playouts */
+  uint64_t cpu_depth_sum;  /* sum of their simulated nodes' depths */
+  uint64_t cpu_nodes;      /* nodes added by CPU iterations */
+  uint64_t gpu_nodes;      /* nodes added by the GPU steps' selections */
+  double select_ms;        /* host time selecting the GPU leaves (the sequential part, L303-L310) */
+  double gpu_ms;           /* host time while the kernel was in flight (CPU iterating) */
+  double backprop_ms;      /* host time backpropagating the kernel's results */
+} mcts_hosted_info;
+
+/* Block parallelism with CPU-managed trees, the paper's own design ("The trees
+ * are still controlled by the CPU threads, GPU simulates only", L302-L303),
+ * and its hybrid CPU-GPU processing (§III-A, Fig. 4): per step the
+ * host threads select one leaf per tree, ONE playout kernel simulates
+ * threads_per_tree playouts from each (streams c0 = tree, c1 = step, c2 =
+ * thread), and while it runs the host threads run UCT iterations with one host
+ * playout each on the SAME trees (streams c0 = tree, c1 = 0x80000000 + the
+ * tree's CPU iteration count, c2 = 0); then the kernel's results are
+ * backpropagated. Selection is R1 with the parent's simulation count (GPU
+ * steps add threads_per_tree, CPU iterations 1); a child whose GPU result is
+ * pending (n = 0) is an unvisited arm, taken first (R18).
+ *   iteration mode: budget.iterations GPU steps, exactly cpu_iters CPU
+ *     iterations per tree per step: deterministic, bit-exact to the oracle;
+ *     cpu_iters = 0 is the MCTS_BLOCK search bit for bit;
+ *   time mode: steps until time_ms; cpu_iters > 0 lets the host iterate while
+ *     each kernel runs (as many as fit), 0 = no CPU iterations.
+ * MCTS_BLOCK handle; n_trees in [1, 2^20]; threads_per_tree a multiple of 32
+ * in [32, 1024]; cpu_threads in [1, 1024] host threads (the caller's thread
+ * included); iteration mode: iterations * (threads_per_tree + cpu_iters)
+ * < 2^26. out (host): root stats summed over trees ([196] counts GPU steps
+ * and CPU iterations; [200] nodes; [201] 0, the host pools are unbounded);
+ * info (host, nullable). Synchronous; single GPU (tree ids 0..n_trees-1). */
+mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                               uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                               uint32_t cpu_iters, uint32_t cpu_threads, mcts_root_stats* out,
+                               mcts_hosted_info* info);
 
 /* Best move from a (merged) stats vector on the host: argmax of visits[0..64],
  * lowest index on ties, -1 if all zero (R8). */

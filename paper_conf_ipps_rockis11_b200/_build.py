@@ -39,7 +39,8 @@ def build(force: bool = False, verbose: bool = False, out: str = None, defines=(
         return LIB
     tmp = target + f".tmp{os.getpid()}"
     cmd = [NVCC, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-Xptxas", "-v",
-           os.path.join(CSRC, "mcts_api.cu"), os.path.join(CSRC, "host_mcts.cpp"), "-o", tmp]
+           os.path.join(CSRC, "mcts_api.cu"), os.path.join(CSRC, "host_mcts.cpp"),
+           os.path.join(CSRC, "hosted.cpp"), "-o", tmp]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + res.stdout + res.stderr)

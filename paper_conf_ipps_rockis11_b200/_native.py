@@ -23,7 +23,7 @@ MCTS_FLAG_CHECK_TREE = 1
 # every symbol include/mcts.h declares
 EXPORTS = (
     "mcts_create", "mcts_destroy", "mcts_playouts", "mcts_playouts_async", "mcts_search",
-    "mcts_search_async", "mcts_search_hybrid", "mcts_best_move", "mcts_perft", "mcts_gen_positions_async", "mcts_ln_table",
+    "mcts_search_async", "mcts_search_hybrid", "mcts_search_hosted", "mcts_playouts_ex_async", "mcts_best_move", "mcts_perft", "mcts_gen_positions_async", "mcts_ln_table",
     "mcts_status_string", "mcts_last_error", "mcts_version",
 )
 
@@ -58,6 +58,12 @@ class RootStats(ctypes.Structure):
                 ("best_move", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
+class HostedInfo(ctypes.Structure):
+    _fields_ = [("steps", ctypes.c_uint64), ("cpu_iterations", ctypes.c_uint64), ("cpu_plies", ctypes.c_uint64),
+                ("cpu_depth_sum", ctypes.c_uint64), ("cpu_nodes", ctypes.c_uint64), ("gpu_nodes", ctypes.c_uint64),
+                ("select_ms", ctypes.c_double), ("gpu_ms", ctypes.c_double), ("backprop_ms", ctypes.c_double)]
+
+
 _lib = None
 
 
@@ -81,6 +87,10 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
     L.mcts_playouts.restype = i32
     L.mcts_playouts_async.argtypes = [vp, vp, u32, u32, u64, u32, vp, vp, vp]
     L.mcts_playouts_async.restype = i32
+    L.mcts_playouts_ex_async.argtypes = [vp, vp, u32, u32, u64, u32, u32, vp, vp, vp]
+    L.mcts_playouts_ex_async.restype = i32
+    L.mcts_search_hosted.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, u32, P(RootStats), P(HostedInfo)]
+    L.mcts_search_hosted.restype = i32
     L.mcts_search.argtypes = [vp, P(Position), Budget, u32, u32, u64, P(RootStats)]
     L.mcts_search.restype = i32
     L.mcts_search_async.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, vp, vp]
@@ -214,6 +224,23 @@ class Mcts:
         d = self._stats_dict(out)
         d["cpu"] = self._stats_dict(cpu)
         return d
+
+    def search_hosted(self, root=None, iterations: int = 0, time_ms: float = 0.0, n_trees: int = 1,
+                      threads_per_tree: int = 64, seed: int = 1, cpu_iters: int = 0, cpu_threads: int = 1) -> dict:
+        """mcts_search_hosted: CPU-managed trees, GPU playouts per step, and cpu_iters
+        host iterations per tree per step on the same trees (Fig. 4)."""
+        out, info = RootStats(), HostedInfo()
+        rp = ctypes.byref(_pos(root)) if root is not None else None
+        self._check(self.L.mcts_search_hosted(self.h, rp, Budget(iterations, time_ms), n_trees, threads_per_tree,
+                                              seed, cpu_iters, cpu_threads, ctypes.byref(out), ctypes.byref(info)))
+        d = self._stats_dict(out)
+        d["info"] = {k: getattr(info, k) for k, _ in HostedInfo._fields_}
+        return d
+
+    def playouts_ex_async(self, d_leaves_ptr: int, n_leaves: int, n_per_leaf: int, seed: int, c0_base: int,
+                          c1: int, d_out_ptr: int, d_plies_ptr: int = 0, stream=None):
+        self._check(self.L.mcts_playouts_ex_async(self.h, d_leaves_ptr, n_leaves, n_per_leaf, seed, c0_base, c1,
+                                                  d_out_ptr, d_plies_ptr or None, _stream_ptr(stream)))
 
     def search_async(self, root, iterations: int, time_ms: float, n_trees: int,
                      threads_per_tree: int, seed: int, tree_id_base: int, d_stats_ptr: int,

@@ -18,6 +18,7 @@
 #include "../../include/mcts.h"
 #include "kernels.cuh"
 #include "host_mcts.h"
+#include "hosted.h"
 
 using namespace mcts_dev;
 
@@ -65,6 +66,12 @@ struct mcts_handle {
   uint32_t work_slot = 0;
   int playout_ctas = 0;       // resident playout CTAs (SMs x occupancy)
   std::vector<double> host_lnT1;  // RN(ln k) for the hybrid's host trees
+
+  // mcts_search_hosted: pinned leaf / result buffers and the step event
+  mcts_position* h_pin_leaves = nullptr;
+  mcts_wdl* h_pin_wdl = nullptr;
+  size_t pin_cap = 0;
+  cudaEvent_t step_event = nullptr;
 };
 
 namespace {
@@ -438,6 +445,68 @@ void fill_root_stats(const long long* hs, mcts_root_stats* out) {
   out->reserved = 0;
 }
 
+// Host ln table lnT[k] = RN(ln k) for k <= K (unit 1) for the host-side trees,
+// generated by the device ln kernel (the host has no correctly rounded ln).
+mcts_status ensure_host_lnT1(mcts_handle* h, uint64_t K) {
+  if (h->host_lnT1.size() >= K + 1) return MCTS_OK;
+  double* d = nullptr;
+  const size_t n = (size_t)K + 1;
+  CK(h, cudaMalloc(&d, n * sizeof(double)));
+  ln_table_kernel<<<(unsigned)((n + 255) / 256), 256, 0, h->stream>>>(d, 1u, (u32)K);
+  std::vector<double> tmp(n);
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(tmp.data(), d, n * sizeof(double), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  cudaFree(d);
+  if (e != cudaSuccess) return cuda_fail(h, e, "host ln table");
+  h->host_lnT1.swap(tmp);
+  return MCTS_OK;
+}
+
+// The GPU side of mcts_search_hosted (hosted.h Gpu): one async step on the
+// handle's stream — leaves H2D, the playouts kernel (c1 = step), W/D/L D2H.
+struct HostedGpu {
+  mcts_handle* h;
+  uint64_t seed;
+  uint32_t unit;
+  mcts_position* d_leaves;
+  mcts_wdl* d_wdl;
+  unsigned long long* d_plies;
+  cudaError_t err;
+};
+
+int hosted_submit(void* ctx, uint32_t n, uint32_t step) {
+  HostedGpu* g = (HostedGpu*)ctx;
+  mcts_handle* h = g->h;
+  cudaStream_t s = h->stream;
+  cudaError_t e = cudaMemcpyAsync(g->d_leaves, h->h_pin_leaves, (size_t)n * sizeof(mcts_position),
+                                  cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess &&
+      mcts_playouts_ex_async(h, g->d_leaves, n, g->unit, g->seed, 0u, step, g->d_wdl, (uint64_t*)g->d_plies, s))
+    e = cudaErrorLaunchFailure;
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(h->h_pin_wdl, g->d_wdl, (size_t)n * sizeof(mcts_wdl), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaEventRecord(h->step_event, s);
+  g->err = e;
+  return e == cudaSuccess ? 0 : -1;
+}
+
+int hosted_done(void* ctx) {
+  HostedGpu* g = (HostedGpu*)ctx;
+  const cudaError_t e = cudaEventQuery(g->h->step_event);
+  if (e == cudaSuccess) return 1;
+  if (e == cudaErrorNotReady) return 0;
+  g->err = e;
+  return -1;
+}
+
+int hosted_wait(void* ctx) {
+  HostedGpu* g = (HostedGpu*)ctx;
+  const cudaError_t e = cudaEventSynchronize(g->h->step_event);
+  if (e != cudaSuccess) { g->err = e; return -1; }
+  return 0;
+}
+
 }  // namespace
 
 extern "C" {
@@ -531,13 +600,16 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
+  if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
+  if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
+  if (h->step_event) cudaEventDestroy(h->step_event);
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
 
-mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
-                                uint32_t n_per_leaf, uint64_t seed, uint32_t leaf_id_base,
-                                mcts_wdl* d_out, uint64_t* d_plies, void* stream) {
+mcts_status mcts_playouts_ex_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
+                                   uint32_t n_per_leaf, uint64_t seed, uint32_t c0_base, uint32_t c1,
+                                   mcts_wdl* d_out, uint64_t* d_plies, void* stream) {
   if (!h) return MCTS_E_INVALID_ARGUMENT;
   if (n_leaves && (!d_leaves || !d_out)) return fail(h, MCTS_E_INVALID_ARGUMENT, "NULL leaves / out");
   mcts_status st = check_device(h);
@@ -554,10 +626,17 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
   u32* work = h->d_work + (h->work_slot++ % kWorkSlots);
   CK(h, cudaMemsetAsync(work, 0, sizeof(u32), s));
   playouts_kernel<<<blocks, kPlayoutThreads, 0, s>>>(
-      (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), leaf_id_base, (WdlOut*)d_out,
+      (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), c0_base, c1, (WdlOut*)d_out,
       (unsigned long long*)d_plies, h->d_rays, work);
   CK(h, cudaGetLastError());
   return MCTS_OK;
+}
+
+mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
+                                uint32_t n_per_leaf, uint64_t seed, uint32_t leaf_id_base,
+                                mcts_wdl* d_out, uint64_t* d_plies, void* stream) {
+  return mcts_playouts_ex_async(h, d_leaves, n_leaves, n_per_leaf, seed, leaf_id_base, 0u, d_out, d_plies,
+                                stream);
 }
 
 mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
@@ -644,20 +723,8 @@ mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_b
     return fail(h, MCTS_E_INVALID_ARGUMENT, "iterations must be in [1, 2^24]");
   mcts_status st = check_device(h);
   if (st) return st;
-  // Host ln table lnT[k] = RN(ln k) (unit = 1), generated by the device kernel.
-  if (h->host_lnT1.size() < host_k + 1) {
-    double* d = nullptr;
-    const size_t n = (size_t)host_k + 1;
-    CK(h, cudaMalloc(&d, n * sizeof(double)));
-    ln_table_kernel<<<(unsigned)((n + 255) / 256), 256, 0, h->stream>>>(d, 1u, (u32)host_k);
-    std::vector<double> tmp(n);
-    cudaError_t e = cudaGetLastError();
-    if (e == cudaSuccess) e = cudaMemcpyAsync(tmp.data(), d, n * sizeof(double), cudaMemcpyDeviceToHost, h->stream);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
-    cudaFree(d);
-    if (e != cudaSuccess) return cuda_fail(h, e, "host ln table");
-    h->host_lnT1.swap(tmp);
-  }
+  st = ensure_host_lnT1(h, host_k);
+  if (st) return st;
   // GPU trees (async), then the host trees in this thread's pool while the
   // kernel runs; host tree ids start at 0x40000000 so no stream is shared.
   st = search_impl(h, rp, budget, n_trees, threads_per_tree, seed, 0, h->d_stats, h->stream);
@@ -686,6 +753,101 @@ mcts_status mcts_search_hybrid(mcts_handle* h, const mcts_position* root, mcts_b
   if (out_cpu) fill_root_stats(cs, out_cpu);
   for (int i = 0; i < MCTS_STATS_LEN; ++i) hs[i] += cs[i];  // root sum over all trees (L199-L202)
   fill_root_stats(hs, out);
+  return MCTS_OK;
+}
+
+mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_budget budget,
+                               uint32_t n_trees, uint32_t threads_per_tree, uint64_t seed,
+                               uint32_t cpu_iters, uint32_t cpu_threads, mcts_root_stats* out,
+                               mcts_hosted_info* info) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (!out) return fail(h, MCTS_E_INVALID_ARGUMENT, "out == NULL");
+  if (h->params.scheme != MCTS_BLOCK) return fail(h, MCTS_E_INVALID_ARGUMENT, "hosted search needs an MCTS_BLOCK handle");
+  const mcts_position* rp = root ? root : (h->has_position ? &h->position : nullptr);
+  if (!rp) return fail(h, MCTS_E_INVALID_ARGUMENT, "no root position");
+  if (!position_ok(*rp)) return fail(h, MCTS_E_INVALID_POSITION, "root: black & white overlap or bad to_move");
+  const bool by_iter = budget.iterations != 0, by_time = budget.time_ms != 0.0;
+  if (by_iter == by_time) return fail(h, MCTS_E_INVALID_ARGUMENT, "budget: exactly one of iterations / time_ms must be non-zero");
+  if (by_time && !(budget.time_ms > 0.0 && budget.time_ms < 3.6e6))
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "budget.time_ms must be in (0, 3.6e6)");
+  if (n_trees == 0 || n_trees > (1u << 20)) return fail(h, MCTS_E_INVALID_ARGUMENT, "n_trees must be in [1, 2^20]");
+  if (threads_per_tree == 0 || threads_per_tree % 32 || threads_per_tree > 1024)
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "threads_per_tree must be a multiple of 32 in [32, 1024]");
+  if (cpu_threads == 0 || cpu_threads > 1024) return fail(h, MCTS_E_INVALID_ARGUMENT, "cpu_threads must be in [1, 1024]");
+  uint64_t K;  // largest parent simulation count a selection can see
+  if (by_iter) {
+    const uint64_t per = (uint64_t)threads_per_tree + cpu_iters;
+    if (budget.iterations >= (1ull << 26) || budget.iterations * per >= (1ull << 26))
+      return fail(h, MCTS_E_INVALID_ARGUMENT, "iterations * (threads_per_tree + cpu_iters) must be < 2^26");
+    K = budget.iterations * per + 2;
+  } else {
+    K = 1ull << 22;
+  }
+  mcts_status st = check_device(h);
+  if (st) return st;
+  st = ensure_host_lnT1(h, K);
+  if (st) return st;
+  if (h->pin_cap < n_trees) {
+    if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
+    if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
+    h->h_pin_leaves = nullptr; h->h_pin_wdl = nullptr; h->pin_cap = 0;
+    CK(h, cudaHostAlloc((void**)&h->h_pin_leaves, (size_t)n_trees * sizeof(mcts_position), cudaHostAllocDefault));
+    CK(h, cudaHostAlloc((void**)&h->h_pin_wdl, (size_t)n_trees * sizeof(mcts_wdl), cudaHostAllocDefault));
+    h->pin_cap = n_trees;
+  }
+  if (!h->step_event) CK(h, cudaEventCreateWithFlags(&h->step_event, cudaEventDisableTiming));
+  void* p = h->d_leaves;
+  st = ensure(h, &p, &h->leaves_cap, (size_t)n_trees * sizeof(DevPosition));
+  if (st) return st;
+  h->d_leaves = (DevPosition*)p;
+  p = h->d_wdl;
+  st = ensure(h, &p, &h->wdl_cap, (size_t)n_trees * sizeof(WdlOut));
+  if (st) return st;
+  h->d_wdl = (WdlOut*)p;
+  CK(h, cudaMemsetAsync(h->d_plies, 0, sizeof(unsigned long long), h->stream));
+
+  HostedGpu g{h, seed, threads_per_tree, (mcts_position*)h->d_leaves, (mcts_wdl*)h->d_wdl, h->d_plies, cudaSuccess};
+  mcts_hosted::Gpu gpu{&g, hosted_submit, hosted_done, hosted_wait,
+                       (mcts_hosted::LeafRec*)h->h_pin_leaves, (const mcts_hosted::WdlRec*)h->h_pin_wdl};
+  mcts_hosted::Args a;
+  a.own = rp->to_move ? rp->white : rp->black;
+  a.opp = rp->to_move ? rp->black : rp->white;
+  a.seed = seed;
+  a.C = h->params.c_uct;
+  a.n_trees = n_trees;
+  a.tree_id_base = 0;
+  a.unit = threads_per_tree;
+  a.steps = by_iter ? budget.iterations : ~0ull;
+  a.cpu_iters = cpu_iters;
+  a.deadline_ns = by_time ? std::chrono::steady_clock::now().time_since_epoch().count() +
+                                (int64_t)llround(budget.time_ms * 1e6)
+                          : 0;
+  a.threads = cpu_threads;
+  a.lnT = h->host_lnT1.data();
+  a.lnT_size = h->host_lnT1.size();
+  long long hs[MCTS_STATS_LEN];
+  mcts_hosted::Info hi;
+  const int r = mcts_hosted::run(a, gpu, (int64_t*)hs, &hi);
+  if (r < 0) {
+    cudaStreamSynchronize(h->stream);
+    return cuda_fail(h, g.err == cudaSuccess ? cudaErrorUnknown : g.err, "mcts_search_hosted: GPU step");
+  }
+  unsigned long long gpu_plies = 0;
+  CK(h, cudaMemcpyAsync(&gpu_plies, h->d_plies, sizeof(gpu_plies), cudaMemcpyDeviceToHost, h->stream));
+  CK(h, cudaStreamSynchronize(h->stream));
+  hs[197] += (long long)gpu_plies;
+  fill_root_stats(hs, out);
+  if (info) {
+    info->steps = hi.steps;
+    info->cpu_iterations = hi.cpu_iterations;
+    info->cpu_plies = hi.cpu_plies;
+    info->cpu_depth_sum = hi.cpu_depth_sum;
+    info->cpu_nodes = hi.cpu_nodes;
+    info->gpu_nodes = hi.gpu_nodes;
+    info->select_ms = hi.select_ms;
+    info->gpu_ms = hi.gpu_ms;
+    info->backprop_ms = hi.backprop_ms;
+  }
   return MCTS_OK;
 }
 

@@ -25,7 +25,9 @@ struct WdlOut {  // layout of mcts_wdl
 // (dynamic balancing; the per-CTA ray table is loaded once). Playout g of a
 // launch is playout j = g mod n_per_leaf of leaf g / n_per_leaf (leaf-major, so
 // a warp's 32 lanes usually share a leaf and finish within a ply or two of each
-// other). Outcomes are reduced per (warp, leaf) with match_any + ballot + popc
+// other); its RNG stream is (c0 = leaf_id_base + leaf, c1, c2 = j) — c1 = 0
+// for mcts_playouts, the step for the CPU-managed trees of mcts_search_hosted.
+// Outcomes are reduced per (warp, leaf) with match_any + ballot + popc
 // and added with one atomic per counter; plies with one atomic per warp.
 // ---------------------------------------------------------------------------
 #ifndef MCTS_PLAYOUT_THREADS
@@ -46,7 +48,7 @@ __device__ __forceinline__ void load_rays(u64* s_rays, const u64* __restrict__ g
 
 __global__ void __launch_bounds__(kPlayoutThreads, MCTS_PLAYOUT_MINB)
 playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_leaf, uint2 key,
-                u32 leaf_id_base, WdlOut* __restrict__ out, unsigned long long* plies_out,
+                u32 leaf_id_base, u32 c1, WdlOut* __restrict__ out, unsigned long long* plies_out,
                 const u64* __restrict__ g_rays, u32* __restrict__ work) {
   __shared__ u64 s_rays[kRayTable];
   load_rays(s_rays, g_rays);
@@ -70,7 +72,7 @@ playouts_kernel(const DevPosition* __restrict__ leaves, u32 n_leaves, u32 n_per_
       const DevPosition p = leaves[leaf];
       const u64 own = p.to_move ? p.white : p.black;
       const u64 opp = p.to_move ? p.black : p.white;
-      r = playout(own, opp, key, leaf_id_base + leaf, 0u, j, s_rays, &plies);
+      r = playout(own, opp, key, leaf_id_base + leaf, c1, j, s_rays, &plies);
     }
     const u32 grp = __match_any_sync(kFullMask, leaf);
     const u32 wins = __popc(__ballot_sync(kFullMask, r == 1) & grp);
