@@ -412,8 +412,9 @@ def selfplay_leg(args, world, rank, local):
     if world > 1:
         init_dist(dist, torch, local)
     hybrid = args.sp_scheme in ("hybrid", "hybrid-tree")
-    if hybrid and world > 1:
-        raise SystemExit("--sp-scheme hybrid is single-GPU")
+    hosted = args.sp_scheme in ("hosted", "hosted-hybrid")
+    if (hybrid or hosted) and world > 1:
+        raise SystemExit("--sp-scheme hybrid / hosted is single-GPU")
     scheme = {"leaf": "leaf", "tree": "tree", "hybrid-tree": "tree"}.get(args.sp_scheme, "block")
     n_trees, threads = SCHEME_SHAPE[scheme]
     m = pkg.Mcts(c_uct=args.c_uct, scheme=scheme, device=local)
@@ -423,6 +424,12 @@ def selfplay_leg(args, world, rank, local):
 
     def search(black, white, to_move, seed):
         pos = pkg.position(black, white, to_move)
+        if hosted:  # NEXT-1: CPU-managed trees, GPU playouts per step (+ CPU iterations meanwhile)
+            r = m.search_hosted(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads, seed=seed,
+                                cpu_iters=1 if args.sp_scheme == "hosted-hybrid" else 0,
+                                cpu_threads=len(os.sched_getaffinity(0)))
+            return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1),
+                    (r["refused_expansions"], r["slots_used"], max(r["slots_used"], 1)))
         if hybrid:  # NEXT-1: GPU trees + one host tree per host core, root sums merged
             r = m.search_hybrid(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads,
                                 seed=seed, cpu_threads=len(os.sched_getaffinity(0)))
@@ -516,6 +523,42 @@ def init_dist(dist, torch, local):
           f"world={dist.get_world_size()} device=cuda:{local}", file=sys.stderr, flush=True)
 
 
+def hosted_leg(m, ms):
+    """The paper's block parallelism as it built it: CPU-managed trees, one GPU
+    playout kernel per step, without and with the hybrid CPU
+    iterations on the same trees while the kernel runs (Fig. 4, P:L312-L339);
+    configs[2] shape from the opening, time mode. Reports playouts/s, the
+    sequential host share of a step and the CPU's share of the
+    iterations, nodes and root visits."""
+    cores = len(os.sched_getaffinity(0))
+    out = {"workload": f"NEXT-1 CPU-managed trees: {SEARCH_TREES} trees x {SEARCH_THREADS} GPU threads, "
+                       f"{ms:.0f} ms, opening root, C=1.0, {cores} host threads"}
+    for name, cpu_iters in (("gpu_only", 0), ("hybrid", 1)):
+        kw = dict(time_ms=ms, n_trees=SEARCH_TREES, threads_per_tree=SEARCH_THREADS, seed=1000,
+                  cpu_iters=cpu_iters, cpu_threads=cores)
+        m.search_hosted(pkg_opening(), **kw)  # warm-up (pinned buffers, ln table)
+        t0 = time.perf_counter()
+        r = m.search_hosted(pkg_opening(), **kw)
+        dt = time.perf_counter() - t0
+        st, inf = r["stats"], r["info"]
+        step_ms = inf["select_ms"] + inf["gpu_ms"] + inf["backprop_ms"]
+        out[name] = {"playouts_per_s": float(st[195]) / dt, "ms": dt * 1e3, "steps": inf["steps"],
+                     "mean_depth": float(st[198]) / max(float(st[196]), 1.0),
+                     "host_select_share": inf["select_ms"] / max(step_ms, 1e-9),
+                     "host_backprop_share": inf["backprop_ms"] / max(step_ms, 1e-9),
+                     "cpu_iteration_share": inf["cpu_iterations"] / max(float(st[196]), 1.0),
+                     "cpu_node_share": inf["cpu_nodes"] / max(inf["cpu_nodes"] + inf["gpu_nodes"], 1),
+                     "cpu_root_visit_share": inf["cpu_iterations"] / max(float(st[195]), 1.0),
+                     "cpu_mean_depth": inf["cpu_depth_sum"] / max(inf["cpu_iterations"], 1),
+                     "best_move": int(r["best_move"])}
+    return out
+
+
+def pkg_opening():
+    import paper_conf_ipps_rockis11_b200 as pkg
+    return pkg.opening()
+
+
 def pool_info(st) -> dict:
     """Node-pool saturation of a search (stats [199]-[201], include/mcts.h)."""
     return {"refused_expansions": int(st[199]), "pool_slots_used": int(st[200]),
@@ -542,7 +585,8 @@ def main():
     ap.add_argument("--selfplay", type=int, default=0,
                     help="play N games vs the CPU oracle MCTS and print the win%% line instead")
     ap.add_argument("--move-ms", type=float, default=SEARCH_MS, help="self-play time per move")
-    ap.add_argument("--sp-scheme", default="block", choices=["block", "leaf", "hybrid", "tree", "hybrid-tree"])
+    ap.add_argument("--sp-scheme", default="block",
+                    choices=["block", "leaf", "hybrid", "tree", "hybrid-tree", "hosted", "hosted-hybrid"])
     ap.add_argument("--c-uct", type=float, default=0.25,
                     help="UCB constant C of the GPU searcher (0.25: best of {0.25, 0.5, 1, 2} "
                          "in 10-game self-play at 100 ms per move, profiles/r01_selfplay_c*.json)")
@@ -701,6 +745,7 @@ def main():
     search = None
     leaf_search = None
     tree_search = None
+    hosted_search = None
     launches = args.steps  # one playouts_kernel per timed step (the headline region)
 
     def run_search(handle, n_trees, threads, id_base, it_scale=1):
@@ -763,6 +808,8 @@ def main():
             **pool_info(tt),
         }
         mt.close()
+        if rank == 0:  # NEXT-1: the paper's CPU-managed trees + hybrid CPU work (single GPU)
+            hosted_search = hosted_leg(m, args.search_ms)
 
     log('if sampler is not None:')
     if sampler is not None:
@@ -811,7 +858,7 @@ def main():
         "gpu_launches": launches,
         "clocks": clocks,
         "opening_batch": opening_batch, "search": search, "leaf_search": leaf_search,
-        "tree_search": tree_search,
+        "tree_search": tree_search, "hosted_search": hosted_search,
     }
     log('if not args.no_cpu and world =')
     if not args.no_cpu and world == 1:
