@@ -219,6 +219,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
     init_node(T, 0, own, opp, 0xFFu);
     s_slot_used = 1;
   }
+  __syncthreads();  // the root (global) and s_slot_used before any lane of the leader reads them
   u32 it = 0;
   for (;; ++it) {
     if (leader) {
