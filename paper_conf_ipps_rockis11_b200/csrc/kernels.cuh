@@ -11,6 +11,7 @@
 //   gen_positions_kernel synthetic input recipe
 #pragma once
 #include <cstdint>
+#include <cooperative_groups.h>
 #include "reversi_device.cuh"
 #include "ln_device.cuh"
 #include "tree_device.cuh"
@@ -137,66 +138,42 @@ block_search_kernel(TreePool T, SearchArgs a) {
 // Leaf-parallel UCT: one tree; every thread of the grid
 // plays out from the same leaf each iteration. CTA 0's warp 0 (the leader)
 // owns the tree (select/expand/backprop); all CTAs are co-resident
-// (cooperative launch). One grid-wide hand-off per iteration instead of two
-// barriers:
-//   leader: publishes the iteration's leaf in S, then gen = it + 1 (release);
-//   every CTA: waits for gen > it (acquire), plays its playouts, reduces them
-//     (ballots + shared memory), adds (W, D) to S->wd[it & 1] and then bumps
-//     S->done[it & 1] (fence + atomic: release);
-//   leader: waits for done[it & 1] == gridDim (acquire), takes and clears the
-//     sums, backpropagates, selects the next leaf and publishes it.
+// (cooperative launch). One grid barrier per iteration (round 1 used two):
+//   leader: collects iteration it - 1 (waits until all gridDim CTAs have
+//     posted, takes and clears the sums), backpropagates, selects iteration
+//     it's leaf and writes it to S;
+//   grid.sync(): the leaf is published;
+//   every CTA: plays its playouts, reduces them (ballots + shared memory),
+//     adds (W, D) to S->wd[it & 1] and bumps S->done[it & 1] (fence + atomic),
+//     then goes straight to the next grid.sync.
 // The parity double-buffer makes the clears safe: slot it & 1 is next written
-// in iteration it + 2, which no CTA reaches before the leader publishes it.
-// Only the leader touches the tree, so its reads never see another SM's stale
-// L1 lines; the hand-off words are read with L2 (.cg / acquire) loads.
+// in iteration it + 2, after two more grid barriers. Only the leader touches
+// the tree; the sums and the leaf are read with L2 (.cg / acquire) loads.
 // ---------------------------------------------------------------------------
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
-  u32 gen;          // iterations whose leaf has been published
-  u32 done[2];      // CTAs finished with iteration it (parity it & 1)
+  u32 done[2];      // CTAs that posted iteration it (parity it & 1)
   u32 wd[2][2];     // per-iteration-parity wins, draws
+  u32 abort;        // watchdog: the leader's wait exceeded kLeafWaitNs (diag below)
+  u32 diag[4];      // iteration, count seen, gridDim, 0
 };
+
+// The leader's wait never legitimately exceeds one playout phase
+// (microseconds); past this the kernel aborts (mcts_search reports
+// MCTS_E_CUDA with the diag) instead of hanging the GPU.
+constexpr u64 kLeafWaitNs = 2000000000ULL;
 
 __device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
   u32 v;
   asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void st_release_u32(u32* p, u32 v) {
-  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// The leader warp selects iteration `it`'s leaf (or decides to stop) and
-// publishes it: S fields, then gen = it + 1 with release semantics.
-__device__ __forceinline__ void leaf_select_publish(const TreePool& T, const SearchArgs& a, LeafSync* S,
-                                                    u32* path, u32* slot_used, int* s_depth, u32 it,
-                                                    u64 deadline, int lane, unsigned long long& depth_sum,
-                                                    unsigned long long& refused) {
-  u32 stop = 0;
-  if (lane == 0) {
-    stop = meta_term(T.meta[0]) || it >= a.max_iterations;
-    if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
-  }
-  stop = __shfl_sync(kFull, stop, 0);
-  if (!stop) {
-    const LeafInfo L = select_expand(T, 0, path, slot_used, a.lnT, a.unit, a.C, lane);
-    if (lane == 0) {
-      *s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
-      depth_sum += (unsigned)L.depth;
-      refused += L.refused;
-    }
-  }
-  if (lane == 0) {
-    S->stop = stop;
-    __threadfence();
-    st_release_u32(&S->gen, it + 1u);
-  }
-  __syncwarp();
-}
 
 __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
   __shared__ u32 path[kMaxPath];
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
@@ -209,35 +186,55 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   const u32 unit = a.unit;
   const u32 G = gridDim.x;
   const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
-  u32 plies = 0;
-  unsigned long long depth_sum = 0;  // leader lane 0
-  unsigned long long refused = 0;    // leader lane 0
-
-  if (leader && lane == 0) {
+  if (blockIdx.x == 0 && tid == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
     const u64 opp = a.root.to_move ? a.root.black : a.root.white;
     init_node(T, 0, own, opp, 0xFFu);
     s_slot_used = 1;
   }
-  __syncthreads();  // the root (global) and s_slot_used before any lane of the leader reads them
+  __syncthreads();
+  u32 plies = 0;
   u32 it = 0;
+  unsigned long long depth_sum = 0;  // leader lane 0
+  unsigned long long refused = 0;    // leader lane 0
   for (;; ++it) {
     if (leader) {
+      u32 stop = 0;
       if (it > 0) {  // collect iteration it - 1 from every CTA, backpropagate
         const u32 pp = (it - 1u) & 1u;
-        if (lane == 0)
-          while (ld_acquire_u32(&S->done[pp]) < G) __nanosleep(20);
+        if (lane == 0) {
+          const u64 t0 = globaltimer_ns();
+          u32 v;
+          while ((v = ld_acquire_u32(&S->done[pp])) < G) {
+            __nanosleep(20);
+            if (globaltimer_ns() - t0 > kLeafWaitNs) {
+              S->abort = 1u; S->diag[0] = it; S->diag[1] = v; S->diag[2] = G; S->diag[3] = 0;
+              break;
+            }
+          }
+        }
         __syncwarp();
         const u32 W = __ldcg(&S->wd[pp][0]), D = __ldcg(&S->wd[pp][1]);
         __syncwarp();
         if (lane == 0) { S->wd[pp][0] = 0; S->wd[pp][1] = 0; S->done[pp] = 0; }
         backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
       }
-      leaf_select_publish(T, a, S, path, &s_slot_used, &s_depth, it, deadline, lane, depth_sum, refused);
+      if (lane == 0) {
+        stop = S->abort || meta_term(T.meta[0]) || it >= a.max_iterations;
+        if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
+      }
+      stop = __shfl_sync(kFull, stop, 0);
+      if (!stop) {
+        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
+        if (lane == 0) {
+          s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
+          depth_sum += (unsigned)L.depth;
+          refused += L.refused;
+        }
+      }
+      if (lane == 0) S->stop = stop;
     }
-    if (tid == 0)
-      while (ld_acquire_u32(&S->gen) <= it) __nanosleep(32);
-    __syncthreads();
+    grid.sync();
     const u32 stop = __ldcg(&S->stop);
     if (stop) break;
     const u64 own = __ldcg(&S->own), opp = __ldcg(&S->opp);
@@ -261,6 +258,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       atomicAdd(&S->done[par], 1u);
     }
   }
+  if (leader && lane == 0 && S->abort) *a.error = 4;
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
   if (leader && lane == 0 && depth_sum)
