@@ -230,8 +230,9 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
   u64 s = 0;
   for (; s < a.steps; ++s) {
     if (timed && now_ns() >= a.deadline_ns) break;
-    // the ln table covers every parent count this step can reach
-    if (P.max_root_n.load() + 2ull * a.unit + (timed ? 1000000ull : (u64)a.cpu_iters) + 1 >= a.lnT_size) break;
+    // the ln table covers every parent count this step's selections can read
+    // (at most the root's count plus the CPU iterations of the step)
+    if (P.max_root_n.load() + (timed ? 1000000ull : (u64)a.cpu_iters) >= a.lnT_size) break;
     const int64_t t0 = now_ns();
     phase(kSelect);
     const int64_t t1 = now_ns();
