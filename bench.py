@@ -366,11 +366,19 @@ def h2h_leg(args, local):
     stream = torch.cuda.current_stream()
     st = torch.zeros(STATS_LEN, dtype=torch.int64, device="cuda")
     a, b = args.h2h_schemes.split(",")
-    ha = pkg.Mcts(c_uct=args.c_uct, scheme=a, device=local)
-    hb = pkg.Mcts(c_uct=args.c_uct, scheme=b, device=local)
+    base = {"hosted": "block", "hosted-hybrid": "block"}
+    ha = pkg.Mcts(c_uct=args.c_uct, scheme=base.get(a, a), device=local)
+    hb = pkg.Mcts(c_uct=args.c_uct, scheme=base.get(b, b), device=local)
+    cores = len(os.sched_getaffinity(0))
 
-    def mover(h, n_trees, threads):
+    def mover(h, n_trees, threads, name):
         def move(black, white, to_move, seed):
+            if name in base:  # NEXT-1: CPU-managed trees (+ CPU iterations on them for hosted-hybrid)
+                r = h.search_hosted(pkg.position(black, white, to_move), time_ms=args.move_ms, n_trees=n_trees,
+                                    threads_per_tree=threads, seed=seed,
+                                    cpu_iters=1 if name == "hosted-hybrid" else 0, cpu_threads=cores)
+                return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1),
+                        (0, r["slots_used"], max(r["slots_used"], 1)))
             h.search_async(pkg.position(black, white, to_move), 0, args.move_ms, n_trees, threads, seed, 0,
                            st.data_ptr(), stream)
             torch.cuda.synchronize()
@@ -379,15 +387,18 @@ def h2h_leg(args, local):
                     (int(x[199]), int(x[200]), int(x[201])))
         return move
 
-    r = play_match(mover(ha, *SCHEME_SHAPE[a]), 0, args.selfplay, args.move_ms, tag="h2h",
-                   opp_move=mover(hb, *SCHEME_SHAPE[b]))
+    r = play_match(mover(ha, *SCHEME_SHAPE[base.get(a, a)], a), 0, args.selfplay, args.move_ms, tag="h2h",
+                   opp_move=mover(hb, *SCHEME_SHAPE[base.get(b, b)], b))
     r[f"{a}_playouts_per_move"] = r.pop("gpu_playouts_per_move")
     r[f"{b}_playouts_per_move"] = r.pop("cpu_playouts_per_move")
     r[f"{a}_depth_per_step"] = r.pop("gpu_depth_per_step")
     r[f"{b}_depth_per_step"] = r.pop("opp_depth_per_step")
-    names = {"block": "block parallelism", "leaf": "leaf parallelism", "tree": "tree parallelism"}
+    names = {"block": "block parallelism", "leaf": "leaf parallelism", "tree": "tree parallelism",
+             "hosted": "CPU-managed block parallelism", "hosted-hybrid": "CPU-managed block parallelism + CPU iterations"}
     shape = {k: f"{SCHEME_DESC[k]}: {v[0]} {'workers' if k == 'tree' else 'trees'} x {v[1]} threads"
              for k, v in SCHEME_SHAPE.items()}
+    for k in base:
+        shape[k] = f"NEXT-1 {k} (DESIGN.md §14): {SEARCH_TREES} trees x {SEARCH_THREADS} GPU threads, {cores} host threads"
     print(json.dumps({"metric": f"win% of {names[a]} vs {names[b]} (equal wall time per move)",
                       "value": r["win_pct"], "unit": "%", "n_gpus": 1,
                       "config": {a: shape[a], b: shape[b], "move_ms": args.move_ms, "colours": "alternating",
@@ -598,7 +609,7 @@ def main():
     ap.add_argument("--h2h", action="store_true",
                     help="with --selfplay: head-to-head of two device searchers on one GPU (--h2h-schemes)")
     ap.add_argument("--h2h-schemes", default="block,leaf",
-                    help="A,B of block|leaf|tree (default block,leaf = configs[2] vs configs[3])")
+                    help="A,B of block|leaf|tree|hosted|hosted-hybrid (default block,leaf = configs[2] vs configs[3])")
     ap.add_argument("--fig7", action="store_true", help="with --selfplay: CPU side on 1, 2, 4, ... threads")
     ap.add_argument("--sweep", action="store_true", help="Fig. 5 analog: playouts/s vs GPU threads")
     ap.add_argument("--sweep-games", type=int, default=0,
