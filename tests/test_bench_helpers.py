@@ -159,3 +159,26 @@ def test_self_launch_cmd():
 
 def test_kernel_source_hash_is_stable():
     assert bench.kernel_source_hash() == bench.kernel_source_hash() and len(bench.kernel_source_hash()) == 16
+
+
+def test_play_match_pool_saturation_bookkeeping():
+    """Movers may report (refused expansions, slots used, capacity) per search;
+    play_match sums the refusals and keeps the fullest pool over the games."""
+    import oracle
+    calls = []
+
+    def lowest(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        m = oracle.legal(own, opp)
+        calls.append(seed)
+        return (m & -m).bit_length() - 1, 1, 2.0, (len(calls) % 3, len(calls), 1000)
+
+    def highest(black, white, to_move, seed):
+        own, opp = (black, white) if to_move == 0 else (white, black)
+        return oracle.legal(own, opp).bit_length() - 1, 2
+
+    r = bench.play_match(lowest, 0, 2, 1.0, opp_move=highest)
+    n = len(calls)
+    assert r["gpu_refused_expansions"] == sum(i % 3 for i in range(1, n + 1))
+    assert abs(r["gpu_pool_max_fill"] - n / 1000) < 1e-12
+    assert r["gpu_depth_per_step"] and all(v == 2.0 for v in r["gpu_depth_per_step"].values())
