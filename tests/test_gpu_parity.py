@@ -438,3 +438,21 @@ def test_time_mode_rejects_non_resident_grid(mcts, orc):
     # iteration mode runs any grid (CTAs simply queue)
     res = mcts.search(pkg.opening(), iterations=2, n_trees=148 * 20, threads_per_tree=32, seed=1)
     assert res["iterations"] == 2 * 148 * 20
+
+
+def test_playouts_pinned_host_buffers_graph_path(mcts, orc):
+    """mcts_playouts with pinned host buffers runs as one cached CUDA graph per
+    (buffers, sizes); repeated calls, a seed change (patched kernel node) and a
+    second buffer pair all stay bit-exact, with the ply counts."""
+    n, per = 300, 40
+    leaves = orc.gen_positions(81, n, 20, 40)
+    h_in = torch.from_numpy(leaves.view(np.int64).reshape(-1, 3).copy()).pin_memory()
+    h_out = torch.zeros((n, 3), dtype=torch.int32).pin_memory()
+    for seed in (5, 5, 6, 5):
+        plies = mcts.playouts_host_ptr(h_in.data_ptr(), n, per, seed, h_out.data_ptr())
+        want, wplies = orc.playouts(leaves, per, seed=seed)
+        assert (h_out.numpy() == want).all() and plies == wplies, seed
+    h_out2 = torch.zeros((n, 3), dtype=torch.int32).pin_memory()
+    plies = mcts.playouts_host_ptr(h_in.data_ptr(), n, 7, 9, h_out2.data_ptr())
+    want, wplies = orc.playouts(leaves, 7, seed=9)
+    assert (h_out2.numpy() == want).all() and plies == wplies
