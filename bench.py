@@ -377,8 +377,7 @@ def h2h_leg(args, local):
                 r = h.search_hosted(pkg.position(black, white, to_move), time_ms=args.move_ms, n_trees=n_trees,
                                     threads_per_tree=threads, seed=seed,
                                     cpu_iters=1 if name == "hosted-hybrid" else 0, cpu_threads=cores)
-                return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1),
-                        (0, r["slots_used"], max(r["slots_used"], 1)))
+                return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1))
             h.search_async(pkg.position(black, white, to_move), 0, args.move_ms, n_trees, threads, seed, 0,
                            st.data_ptr(), stream)
             torch.cuda.synchronize()
@@ -439,8 +438,7 @@ def selfplay_leg(args, world, rank, local):
             r = m.search_hosted(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads, seed=seed,
                                 cpu_iters=1 if args.sp_scheme == "hosted-hybrid" else 0,
                                 cpu_threads=len(os.sched_getaffinity(0)))
-            return (r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1),
-                    (r["refused_expansions"], r["slots_used"], max(r["slots_used"], 1)))
+            return r["best_move"], r["root_visits"], r["depth_sum"] / max(r["iterations"], 1)  # host pools: unbounded
         if hybrid:  # NEXT-1: GPU trees + one host tree per host core, root sums merged
             r = m.search_hybrid(pos, time_ms=args.move_ms, n_trees=n_trees, threads_per_tree=threads,
                                 seed=seed, cpu_threads=len(os.sched_getaffinity(0)))

@@ -203,7 +203,10 @@ mcts_status check_device(mcts_handle* h) {
 uint32_t auto_slot_cap(mcts_handle* h, double time_ms, uint32_t n_trees, bool shared) {
   size_t free_b = 0, total_b = 0;
   if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) free_b = (size_t)8 << 30;
-  const double per_ms = shared ? 20000.0 : 100.0;  // measured: ~15k/ms shared tree, ~66/ms per block tree
+  // measured at 500 ms: ~15k/ms for the shared tree from the opening, up to ~3x
+  // that late in a game (short playouts; r2h self-play filled 85% of 2^27 and
+  // refused 319 expansions); ~66/ms per block tree, a few hundred late
+  const double per_ms = shared ? 50000.0 : 100.0;
   double want = time_ms * per_ms * 10.0;
   const double hi = shared ? (double)(1u << 28) : (double)(1u << 24);
   if (want < 65536.0) want = 65536.0;
