@@ -39,6 +39,7 @@ struct PlayoutGraph {
   void* hout = nullptr;
   uint32_t n = 0, per = 0;
   uint64_t seed = 0, last_use = 0;
+  cudaGraph_t graph = nullptr;  // kept: the kernel node is patched through it (cudaGraphExecKernelNodeSetParams)
   cudaGraphExec_t exec = nullptr;
   cudaGraphNode_t knode = nullptr;
   void* d_leaves = nullptr;
@@ -116,6 +117,7 @@ mcts_status fail(mcts_handle* h, mcts_status st, const std::string& msg) {
 }
 
 mcts_status cuda_fail(mcts_handle* h, cudaError_t e, const char* where) {
+  cudaGetLastError();  // a reported (non-sticky) error must not leak into later calls
   std::string msg = std::string(where) + ": " + cudaGetErrorString(e);
   return fail(h, e == cudaErrorMemoryAllocation ? MCTS_E_OOM : MCTS_E_CUDA, msg);
 }
@@ -490,6 +492,7 @@ bool is_pinned(const void* p) {
 
 void free_graph(PlayoutGraph* g) {
   if (g->exec) cudaGraphExecDestroy(g->exec);
+  if (g->graph) cudaGraphDestroy(g->graph);
   cudaFree(g->d_leaves);
   cudaFree(g->d_io);
   if (g->h_plies) cudaFreeHost(g->h_plies);
@@ -521,8 +524,8 @@ mcts_status build_playout_graph(mcts_handle* h, PlayoutGraph* g, int playout_cta
   const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
   const unsigned blocks = (unsigned)(need < (uint64_t)playout_ctas ? need : (uint64_t)playout_ctas);
 
-  cudaGraph_t graph = nullptr;
-  CK(h, cudaGraphCreate(&graph, 0));
+  CK(h, cudaGraphCreate(&g->graph, 0));
+  cudaGraph_t graph = g->graph;
   cudaGraphNode_t zero = nullptr, h2d = nullptr, d2h = nullptr, d2h2 = nullptr;
   cudaMemsetParams mp = {};
   mp.dst = g->d_io;
@@ -548,7 +551,6 @@ mcts_status build_playout_graph(mcts_handle* h, PlayoutGraph* g, int playout_cta
     e = cudaGraphAddMemcpyNode1D(&d2h2, graph, &g->knode, 1, g->h_plies, g->d_io + plies_off,
                                  sizeof(unsigned long long), cudaMemcpyDeviceToHost);
   if (e == cudaSuccess) e = cudaGraphInstantiate(&g->exec, graph, 0);
-  cudaGraphDestroy(graph);
   if (e != cudaSuccess) return cuda_fail(h, e, "mcts_playouts: graph");
   return MCTS_OK;
 }
@@ -649,6 +651,7 @@ mcts_status mcts_create(const mcts_position* position, const mcts_params* params
   if (position && !position_ok(*position))
     return fail(nullptr, MCTS_E_INVALID_POSITION, "position: black & white overlap or bad to_move");
   int ndev = 0;
+  cudaGetLastError();  // a stale error of an earlier, unrelated runtime call is not ours
   cudaError_t e = cudaGetDeviceCount(&ndev);
   if (e != cudaSuccess || ndev == 0)
     return fail(nullptr, MCTS_E_NO_DEVICE, std::string("no CUDA device: ") + cudaGetErrorString(e));
@@ -708,13 +711,8 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
-  for (PlayoutGraph* g : h->graphs) {
-    if (g->exec) cudaGraphExecDestroy(g->exec);
-    cudaFree(g->d_leaves);
-    cudaFree(g->d_io);
-    if (g->h_plies) cudaFreeHost(g->h_plies);
-    delete g;
-  }
+  for (PlayoutGraph* g : h->graphs) free_graph(g);
+  h->graphs.clear();
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
   if (h->step_event) cudaEventDestroy(h->step_event);
@@ -946,14 +944,7 @@ mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_b
   st = ensure_host_lnT1(h, K);
   if (st) return st;
   if (h->pin_cap < n_trees) {
-    for (PlayoutGraph* g : h->graphs) {
-    if (g->exec) cudaGraphExecDestroy(g->exec);
-    cudaFree(g->d_leaves);
-    cudaFree(g->d_io);
-    if (g->h_plies) cudaFreeHost(g->h_plies);
-    delete g;
-  }
-  if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
+    if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
     if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
     h->h_pin_leaves = nullptr; h->h_pin_wdl = nullptr; h->pin_cap = 0;
     CK(h, cudaHostAlloc((void**)&h->h_pin_leaves, (size_t)n_trees * sizeof(mcts_position), cudaHostAllocDefault));

@@ -415,7 +415,10 @@ def test_pool_full_is_counted(orc, scheme, n_trees, threads):
     s = res["stats"]
     assert s[199] > 0
     assert s[200] <= s[201] == (n_trees if scheme != "tree" else 1) * 64
-    assert s[195] == res["iterations"] * threads and s[:65].sum() == s[195]
+    assert s[195] == res["iterations"] * threads
+    # a shared-tree worker that finds every root child claimed but unpublished
+    # simulates from the root itself, so only <= holds there
+    assert s[:65].sum() == s[195] if scheme != "tree" else s[:65].sum() <= s[195]
     m.close()
 
 

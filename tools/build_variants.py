@@ -30,11 +30,6 @@ VARIANTS = {
     "t128m10": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=10"],
     "t128m11": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=11"],
     "t64m20": ["MCTS_PLAYOUT_THREADS=64", "MCTS_PLAYOUT_MINB=20"],
-    "ls2m4": ["MCTS_LANE_STREAM=2", "MCTS_PLAYOUT_MINB=4"],
-    "ls4m4": ["MCTS_LANE_STREAM=4", "MCTS_PLAYOUT_MINB=4"],
-    "ls8m4": ["MCTS_LANE_STREAM=8", "MCTS_PLAYOUT_MINB=4"],
-    "ls4": ["MCTS_LANE_STREAM=4"],
-    "ls16m4": ["MCTS_LANE_STREAM=16", "MCTS_PLAYOUT_MINB=4"],
 }
 
 if __name__ == "__main__":
