@@ -136,17 +136,39 @@ block_search_kernel(TreePool T, SearchArgs a) {
 
 // ---------------------------------------------------------------------------
 // Leaf-parallel UCT: one tree; every thread of the grid
-// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree
-// (select/expand/backprop); the leaf is published through a small global
-// struct between two cooperative-groups grid barriers per iteration
-// (select -> sync -> simulate + per-CTA ballot reduce + atomics -> sync).
-// All CTAs are co-resident (cooperative launch).
+// plays out from the same leaf each iteration. CTA 0's warp 0 (the leader)
+// owns the tree (select/expand/backprop); all CTAs are co-resident
+// (cooperative launch). One grid barrier per iteration (round 1 used two):
+//   leader: collects iteration it - 1 (waits until all gridDim CTAs have
+//     posted, takes and clears the sums), backpropagates, selects iteration
+//     it's leaf and writes it to S;
+//   grid.sync(): the leaf is published;
+//   every CTA: plays its playouts, reduces them (ballots + shared memory),
+//     adds (W, D) to S->wd[it & 1] and bumps S->done[it & 1] (fence + atomic),
+//     then goes straight to the next grid.sync.
+// The parity double-buffer makes the clears safe: slot it & 1 is next written
+// in iteration it + 2, after two more grid barriers. Only the leader touches
+// the tree; the sums and the leaf are read with L2 (.cg / acquire) loads.
 // ---------------------------------------------------------------------------
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
+  u32 done[2];      // CTAs that posted iteration it (parity it & 1)
   u32 wd[2][2];     // per-iteration-parity wins, draws
+  u32 abort;        // watchdog: the leader's wait exceeded kLeafWaitNs (diag below)
+  u32 diag[4];      // iteration, count seen, gridDim, 0
 };
+
+// The leader's wait never legitimately exceeds one playout phase
+// (microseconds); past this the kernel aborts (mcts_search reports
+// MCTS_E_CUDA with the diag) instead of hanging the GPU.
+constexpr u64 kLeafWaitNs = 2000000000ULL;
+
+__device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 
 __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
@@ -162,6 +184,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const bool leader = blockIdx.x == 0 && warp == 0;
   const u32 unit = a.unit;
+  const u32 G = gridDim.x;
   const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
   if (blockIdx.x == 0 && tid == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
@@ -176,16 +199,28 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   unsigned long long refused = 0;    // leader lane 0
   for (;; ++it) {
     if (leader) {
-      if (it > 0) {
-        const u32 par = (it - 1) & 1u;
-        const u32 W = S->wd[par][0], D = S->wd[par][1];
+      u32 stop = 0;
+      if (it > 0) {  // collect iteration it - 1 from every CTA, backpropagate
+        const u32 pp = (it - 1u) & 1u;
+        if (lane == 0) {
+          const u64 t0 = globaltimer_ns();
+          u32 v;
+          while ((v = ld_acquire_u32(&S->done[pp])) < G) {
+            __nanosleep(20);
+            if (globaltimer_ns() - t0 > kLeafWaitNs) {
+              S->abort = 1u; S->diag[0] = it; S->diag[1] = v; S->diag[2] = G; S->diag[3] = 0;
+              break;
+            }
+          }
+        }
         __syncwarp();
-        if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
+        const u32 W = __ldcg(&S->wd[pp][0]), D = __ldcg(&S->wd[pp][1]);
+        __syncwarp();
+        if (lane == 0) { S->wd[pp][0] = 0; S->wd[pp][1] = 0; S->done[pp] = 0; }
         backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
       }
-      u32 stop = 0;
       if (lane == 0) {
-        stop = meta_term(T.meta[0]) || it >= a.max_iterations;
+        stop = S->abort || meta_term(T.meta[0]) || it >= a.max_iterations;
         if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
       }
       stop = __shfl_sync(kFull, stop, 0);
@@ -200,10 +235,10 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       if (lane == 0) S->stop = stop;
     }
     grid.sync();
-    const u32 stop = S->stop;
-    const u64 own = S->own, opp = S->opp;
-    const u32 term = S->term;
+    const u32 stop = __ldcg(&S->stop);
     if (stop) break;
+    const u64 own = __ldcg(&S->own), opp = __ldcg(&S->opp);
+    const u32 term = __ldcg(&S->term);
     int r;
     if (term) {
       const int x = __popcll(own), y = __popcll(opp);
@@ -219,9 +254,11 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       const u32 par = it & 1u;
       atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
       atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
+      __threadfence();
+      atomicAdd(&S->done[par], 1u);
     }
-    grid.sync();
   }
+  if (leader && lane == 0 && S->abort) *a.error = 4;
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
   if (leader && lane == 0 && depth_sum)

@@ -77,13 +77,17 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
   u32 v = 0;
   int depth = 0;
   if (lane == 0) path[0] = 0;
-  u32 meta = T.meta[base];
+  // Control values (meta, first child, parent count) are read by lane 0 and
+  // broadcast, so every lane takes the same path through the loop whatever the
+  // memory system returns to each lane's own load (a leaf kernel whose leader
+  // lanes loaded them individually diverged and deadlocked).
+  u32 meta = __shfl_sync(kFull, T.meta[base], 0);
   // Selection (L157-L178): descend while the node is non-terminal and fully expanded.
   // (depth bound: a game has < 128 plies incl. passes; never reached)
   while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta) && depth < kMaxPath - 2) {
     const u32 nch = meta_nchild(meta);
-    const u32 first = T.first[base + v];
-    const double lnp = lnT[T.k[base + v]];
+    const u32 first = __shfl_sync(kFull, T.first[base + v], 0);
+    const double lnp = lnT[__shfl_sync(kFull, T.k[base + v], 0)];
     double best_u = -__longlong_as_double(0x7FF0000000000000LL);  // -inf
     u32 best_i = kNoChild;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
@@ -100,7 +104,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
     v = first + best_i;
     ++depth;
     if (lane == 0) path[depth] = v;
-    meta = T.meta[base + v];
+    meta = __shfl_sync(kFull, T.meta[base + v], 0);
   }
   // Expansion (L179-L182): the lowest-index untried move, or the pass child.
   LeafInfo L;
