@@ -107,10 +107,17 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
                                                        double C, int lane) {
   u32 v = 0;
   int depth = 0;
-  u32 meta = ld_acq(&T.meta[0]);
-  u32 first = ld_rlx(&T.first[0]);
-  u32 kp = ld_rlx(&T.k[0]) + ld_rlx(&T.vl[0]);  // read before our own virtual visit
-  __syncwarp();
+  // lane 0's reads, broadcast: other workers change the root concurrently, so
+  // lanes reading it themselves could disagree and split the warp
+  u32 meta = 0, first = 0, kp = 0;
+  if (lane == 0) {
+    meta = ld_acq(&T.meta[0]);
+    first = ld_rlx(&T.first[0]);
+    kp = ld_rlx(&T.k[0]) + ld_rlx(&T.vl[0]);  // read before our own virtual visit
+  }
+  meta = __shfl_sync(kFull, meta, 0);
+  first = __shfl_sync(kFull, first, 0);
+  kp = __shfl_sync(kFull, kp, 0);
   if (lane == 0) {
     path[0] = 0;
     atomicAdd(&T.vl[0], 1u);
