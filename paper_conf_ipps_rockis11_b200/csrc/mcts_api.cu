@@ -29,34 +29,6 @@ static_assert(sizeof(mcts_wdl) == sizeof(WdlOut), "wdl layout");
 // on different streams of one handle (up to kWorkSlots in flight) never share one.
 constexpr uint32_t kWorkSlots = 256;
 
-// One cached CUDA graph of the synchronous mcts_playouts call for a given
-// (pinned host input, pinned host output, n_leaves, n_per_leaf): zero the
-// outputs, copy the leaves in, the playouts kernel, copy W/D/L and plies out.
-// It owns its device buffers and its work counter; the seed is patched into
-// the kernel node per call.
-struct PlayoutGraph {
-  const void* hin = nullptr;
-  void* hout = nullptr;
-  uint32_t n = 0, per = 0;
-  uint64_t seed = 0, last_use = 0;
-  cudaGraph_t graph = nullptr;  // kept: the kernel node is patched through it (cudaGraphExecKernelNodeSetParams)
-  cudaGraphExec_t exec = nullptr;
-  cudaGraphNode_t knode = nullptr;
-  void* d_leaves = nullptr;
-  unsigned char* d_io = nullptr;          // wdl[n] | plies (u64) | work (u32)
-  unsigned long long* h_plies = nullptr;  // pinned
-  // kernel arguments (their addresses are the node's kernelParams)
-  const mcts_dev::DevPosition* a_leaves;
-  uint32_t a_n, a_per;
-  uint2 a_key;
-  uint32_t a_base, a_c1;
-  mcts_dev::WdlOut* a_out;
-  unsigned long long* a_plies;
-  const mcts_dev::u64* a_rays;
-  uint32_t* a_work;
-  void* params[10];
-};
-
 struct mcts_handle {
   int device = 0;
   mcts_params params{};
@@ -94,10 +66,6 @@ struct mcts_handle {
   uint32_t work_slot = 0;
   int playout_ctas = 0;       // resident playout CTAs (SMs x occupancy)
   std::vector<double> host_lnT1;  // RN(ln k) for the hybrid's host trees
-
-  // mcts_playouts with pinned host buffers: cached CUDA graphs (one launch per call)
-  std::vector<struct PlayoutGraph*> graphs;
-  uint64_t graph_clock = 0;
 
   // mcts_search_hosted: pinned leaf / result buffers and the step event
   mcts_position* h_pin_leaves = nullptr;
@@ -481,80 +449,6 @@ void fill_root_stats(const long long* hs, mcts_root_stats* out) {
   out->reserved = 0;
 }
 
-bool is_pinned(const void* p) {
-  cudaPointerAttributes at;
-  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
-    cudaGetLastError();  // clear the sticky-free error of an unregistered pointer query
-    return false;
-  }
-  return at.type == cudaMemoryTypeHost;
-}
-
-void free_graph(PlayoutGraph* g) {
-  if (g->exec) cudaGraphExecDestroy(g->exec);
-  if (g->graph) cudaGraphDestroy(g->graph);
-  cudaFree(g->d_leaves);
-  cudaFree(g->d_io);
-  if (g->h_plies) cudaFreeHost(g->h_plies);
-  delete g;
-}
-
-// Build the graph of one synchronous playout call (see PlayoutGraph).
-mcts_status build_playout_graph(mcts_handle* h, PlayoutGraph* g, int playout_ctas) {
-  const size_t wdl_bytes = (size_t)g->n * sizeof(WdlOut);
-  const size_t io_bytes = ((wdl_bytes + 7) & ~(size_t)7) + 16;
-  CK(h, cudaMalloc(&g->d_leaves, (size_t)g->n * sizeof(DevPosition)));
-  CK(h, cudaMalloc((void**)&g->d_io, io_bytes));
-  CK(h, cudaHostAlloc((void**)&g->h_plies, sizeof(unsigned long long), cudaHostAllocDefault));
-  const size_t plies_off = (wdl_bytes + 7) & ~(size_t)7;
-  g->a_leaves = (const DevPosition*)g->d_leaves;
-  g->a_n = g->n;
-  g->a_per = g->per;
-  g->a_key = key_of(g->seed);
-  g->a_base = 0;
-  g->a_c1 = 0;
-  g->a_out = (WdlOut*)g->d_io;
-  g->a_plies = (unsigned long long*)(g->d_io + plies_off);
-  g->a_rays = h->d_rays;
-  g->a_work = (uint32_t*)(g->d_io + plies_off + 8);
-  void* pr[10] = {&g->a_leaves, &g->a_n, &g->a_per, &g->a_key, &g->a_base, &g->a_c1,
-                  &g->a_out, &g->a_plies, &g->a_rays, &g->a_work};
-  memcpy(g->params, pr, sizeof(pr));
-  const uint64_t total = (uint64_t)g->n * g->per;
-  const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
-  const unsigned blocks = (unsigned)(need < (uint64_t)playout_ctas ? need : (uint64_t)playout_ctas);
-
-  CK(h, cudaGraphCreate(&g->graph, 0));
-  cudaGraph_t graph = g->graph;
-  cudaGraphNode_t zero = nullptr, h2d = nullptr, d2h = nullptr, d2h2 = nullptr;
-  cudaMemsetParams mp = {};
-  mp.dst = g->d_io;
-  mp.value = 0;
-  mp.elementSize = 1;
-  mp.width = io_bytes;
-  mp.height = 1;
-  cudaError_t e = cudaGraphAddMemsetNode(&zero, graph, nullptr, 0, &mp);
-  if (e == cudaSuccess)
-    e = cudaGraphAddMemcpyNode1D(&h2d, graph, nullptr, 0, g->d_leaves, g->hin, (size_t)g->n * sizeof(DevPosition),
-                                 cudaMemcpyHostToDevice);
-  cudaKernelNodeParams kp = {};
-  kp.func = (void*)playouts_kernel;
-  kp.gridDim = dim3(blocks);
-  kp.blockDim = dim3(kPlayoutThreads);
-  kp.sharedMemBytes = 0;
-  kp.kernelParams = g->params;
-  cudaGraphNode_t deps[2] = {zero, h2d};
-  if (e == cudaSuccess) e = cudaGraphAddKernelNode(&g->knode, graph, deps, 2, &kp);
-  if (e == cudaSuccess)
-    e = cudaGraphAddMemcpyNode1D(&d2h, graph, &g->knode, 1, g->hout, g->d_io, wdl_bytes, cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess)
-    e = cudaGraphAddMemcpyNode1D(&d2h2, graph, &g->knode, 1, g->h_plies, g->d_io + plies_off,
-                                 sizeof(unsigned long long), cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess) e = cudaGraphInstantiate(&g->exec, graph, 0);
-  if (e != cudaSuccess) return cuda_fail(h, e, "mcts_playouts: graph");
-  return MCTS_OK;
-}
-
 // Host ln table lnT[k] = RN(ln k) for k <= K (unit 1) for the host-side trees,
 // generated by the device ln kernel (the host has no correctly rounded ln).
 mcts_status ensure_host_lnT1(mcts_handle* h, uint64_t K) {
@@ -711,8 +605,6 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
-  for (PlayoutGraph* g : h->graphs) free_graph(g);
-  h->graphs.clear();
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
   if (h->step_event) cudaEventDestroy(h->step_event);
@@ -769,43 +661,6 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
   }
   if ((uint64_t)n_leaves * n_per_leaf / 32 > 0xFFFFFFF0ull)
     return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large (>= 2^37 playouts)");
-  if (is_pinned(leaf_batch) && is_pinned(out_counts)) {
-    // pinned host buffers: the whole call is one cached CUDA graph launch
-    PlayoutGraph* g = nullptr;
-    for (PlayoutGraph* x : h->graphs)
-      if (x->hin == leaf_batch && x->hout == out_counts && x->n == n_leaves && x->per == n_per_leaf) g = x;
-    if (!g) {
-      if (h->graphs.size() >= 4) {  // evict the least recently used
-        size_t lru = 0;
-        for (size_t i = 1; i < h->graphs.size(); ++i)
-          if (h->graphs[i]->last_use < h->graphs[lru]->last_use) lru = i;
-        free_graph(h->graphs[lru]);
-        h->graphs.erase(h->graphs.begin() + lru);
-      }
-      g = new PlayoutGraph();
-      g->hin = leaf_batch; g->hout = out_counts; g->n = n_leaves; g->per = n_per_leaf; g->seed = seed;
-      st = build_playout_graph(h, g, h->playout_ctas);
-      if (st) { free_graph(g); return st; }
-      h->graphs.push_back(g);
-    }
-    if (g->seed != seed) {  // patch the key of the kernel node
-      g->seed = seed;
-      g->a_key = key_of(seed);
-      cudaKernelNodeParams kp = {};
-      kp.func = (void*)playouts_kernel;
-      const uint64_t total = (uint64_t)g->n * g->per;
-      const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
-      kp.gridDim = dim3((unsigned)(need < (uint64_t)h->playout_ctas ? need : (uint64_t)h->playout_ctas));
-      kp.blockDim = dim3(kPlayoutThreads);
-      kp.kernelParams = g->params;
-      CK(h, cudaGraphExecKernelNodeSetParams(g->exec, g->knode, &kp));
-    }
-    g->last_use = ++h->graph_clock;
-    CK(h, cudaGraphLaunch(g->exec, h->stream));
-    CK(h, cudaStreamSynchronize(h->stream));
-    if (out_plies) *out_plies = *g->h_plies;
-    return MCTS_OK;
-  }
   void* p = h->d_leaves;
   st = ensure(h, &p, &h->leaves_cap, (size_t)n_leaves * sizeof(DevPosition));
   if (st) return st;

@@ -443,10 +443,10 @@ def test_time_mode_rejects_non_resident_grid(mcts, orc):
     assert res["iterations"] == 2 * 148 * 20
 
 
-def test_playouts_pinned_host_buffers_graph_path(mcts, orc):
-    """mcts_playouts with pinned host buffers runs as one cached CUDA graph per
-    (buffers, sizes); repeated calls, a seed change (patched kernel node) and a
-    second buffer pair all stay bit-exact, with the ply counts."""
+def test_playouts_pinned_host_buffers(mcts, orc):
+    """mcts_playouts with pinned host buffers (the bench's e2e call): repeated
+    calls, a seed change and a second buffer pair stay bit-exact, with the ply
+    counts."""
     n, per = 300, 40
     leaves = orc.gen_positions(81, n, 20, 40)
     h_in = torch.from_numpy(leaves.view(np.int64).reshape(-1, 3).copy()).pin_memory()
