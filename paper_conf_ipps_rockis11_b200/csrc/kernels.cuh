@@ -144,17 +144,23 @@ block_search_kernel(TreePool T, SearchArgs a) {
 //     it's leaf and writes it to S;
 //   grid.sync(): the leaf is published;
 //   every CTA: plays its playouts, reduces them (ballots + shared memory),
-//     adds (W, D) to S->wd[it & 1] and bumps S->done[it & 1] (fence + atomic),
+//     adds (1, W, D) to the packed word S->post[it & 1] with one atomic,
 //     then goes straight to the next grid.sync.
-// The parity double-buffer makes the clears safe: slot it & 1 is next written
-// in iteration it + 2, after two more grid barriers. Only the leader touches
-// the tree; the sums and the leaf are read with L2 (.cg / acquire) loads.
+// The parity double-buffer makes the clears safe: slot it & 1 is next posted
+// to two barriers after the leader clears it. Only the leader touches the
+// tree; it polls the posts with relaxed L2 loads, the CTAs read the leaf with
+// .cg loads.
 // ---------------------------------------------------------------------------
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
-  u32 done[2];      // CTAs that posted iteration it (parity it & 1)
-  u32 wd[2][2];     // per-iteration-parity wins, draws
+  // Per-iteration-parity posts, one 64-bit word each: CTAs that posted in
+  // bits 0-15, wins in bits 16-39, draws in bits 40-63 (unit <= 65536 < 2^24,
+  // gridDim <= 512 < 2^16). A CTA posts with ONE atomic add, so the leader
+  // reads the count and the sums it covers in one load — no fences, no
+  // acquire (which would invalidate the leader SM's L1, where the hot top of
+  // the tree lives).
+  unsigned long long post[2];
   u32 abort;        // watchdog: the leader's wait exceeded kLeafWaitNs (diag below)
   u32 diag[4];      // iteration, count seen, gridDim, 0
 };
@@ -164,9 +170,9 @@ struct LeafSync {
 // MCTS_E_CUDA with the diag) instead of hanging the GPU.
 constexpr u64 kLeafWaitNs = 2000000000ULL;
 
-__device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
-  u32 v;
-  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
 
@@ -202,21 +208,20 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       u32 stop = 0;
       if (it > 0) {  // collect iteration it - 1 from every CTA, backpropagate
         const u32 pp = (it - 1u) & 1u;
+        unsigned long long v = 0;
         if (lane == 0) {
           const u64 t0 = globaltimer_ns();
-          u32 v;
-          while ((v = ld_acquire_u32(&S->done[pp])) < G) {
+          while (((v = ld_relaxed_u64(&S->post[pp])) & 0xFFFFull) < G) {
             __nanosleep(20);
             if (globaltimer_ns() - t0 > kLeafWaitNs) {
-              S->abort = 1u; S->diag[0] = it; S->diag[1] = v; S->diag[2] = G; S->diag[3] = 0;
+              S->abort = 1u; S->diag[0] = it; S->diag[1] = (u32)(v & 0xFFFFull); S->diag[2] = G; S->diag[3] = 0;
               break;
             }
           }
+          S->post[pp] = 0ull;  // next posted to in iteration it + 1, two barriers later
         }
-        __syncwarp();
-        const u32 W = __ldcg(&S->wd[pp][0]), D = __ldcg(&S->wd[pp][1]);
-        __syncwarp();
-        if (lane == 0) { S->wd[pp][0] = 0; S->wd[pp][1] = 0; S->done[pp] = 0; }
+        v = __shfl_sync(kFull, v, 0);
+        const u32 W = (u32)((v >> 16) & 0xFFFFFFull), D = (u32)(v >> 40);
         backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
       }
       if (lane == 0) {
@@ -250,12 +255,9 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
     const u32 bd = __popc(__ballot_sync(kFull, r == 0));
     if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
     __syncthreads();
-    if (tid == 0) {
-      const u32 par = it & 1u;
-      atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
-      atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
-      __threadfence();
-      atomicAdd(&S->done[par], 1u);
+    if (tid == 0) {  // one atomic: the post count and the sums it covers
+      const unsigned long long w = s_w[0] + s_w[1] + s_w[2] + s_w[3], d = s_d[0] + s_d[1] + s_d[2] + s_d[3];
+      atomicAdd(&S->post[it & 1u], 1ull | (w << 16) | (d << 40));
     }
   }
   if (leader && lane == 0 && S->abort) *a.error = 4;
