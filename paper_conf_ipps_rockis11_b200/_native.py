@@ -72,11 +72,12 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_build.LIB):
-        if not build_if_missing:
-            raise FileNotFoundError(f"{_build.LIB} is missing: run __graft_entry__.build()")
+    lib_path = os.environ.get("MCTS_LIB", _build.LIB)  # tooling: a tuning variant (tools/build_variants.py)
+    if not os.path.exists(lib_path):
+        if not build_if_missing or lib_path != _build.LIB:
+            raise FileNotFoundError(f"{lib_path} is missing: run __graft_entry__.build()")
         _build.build()
-    L = ctypes.CDLL(_build.LIB)
+    L = ctypes.CDLL(lib_path)
     vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32
     P = ctypes.POINTER
     L.mcts_create.argtypes = [P(Position), P(Params), P(vp)]

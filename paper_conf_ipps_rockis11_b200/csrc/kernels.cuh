@@ -151,6 +151,101 @@ block_search_kernel(TreePool T, SearchArgs a) {
 // tree; it polls the posts with relaxed L2 loads, the CTAs read the leaf with
 // .cg loads.
 // ---------------------------------------------------------------------------
+#ifndef MCTS_LEAF_BARRIERS
+#define MCTS_LEAF_BARRIERS 1  // 2: round 1's two grid barriers per iteration (tuning comparison)
+#endif
+#if MCTS_LEAF_BARRIERS == 2
+struct LeafSync {  // two-barrier variant
+  u64 own, opp;
+  u32 term, stop;
+  u32 wd[2][2];     // per-iteration-parity wins, draws
+  u32 abort;
+  u32 diag[4];
+};
+
+__global__ void __launch_bounds__(128)
+leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  __shared__ u32 path[kMaxPath];
+  __shared__ u32 s_slot_used;
+  __shared__ int s_depth;
+  __shared__ u32 s_w[4], s_d[4];
+  __shared__ u64 s_rays[kRayTable];
+  load_rays(s_rays, a.rays);
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const bool leader = blockIdx.x == 0 && warp == 0;
+  const u32 unit = a.unit;
+  const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
+  if (blockIdx.x == 0 && tid == 0) {
+    const u64 own = a.root.to_move ? a.root.white : a.root.black;
+    const u64 opp = a.root.to_move ? a.root.black : a.root.white;
+    init_node(T, 0, own, opp, 0xFFu);
+    s_slot_used = 1;
+  }
+  __syncthreads();
+  u32 plies = 0;
+  u32 it = 0;
+  unsigned long long depth_sum = 0;  // leader lane 0
+  unsigned long long refused = 0;    // leader lane 0
+  for (;; ++it) {
+    if (leader) {
+      if (it > 0) {
+        const u32 par = (it - 1) & 1u;
+        const u32 W = S->wd[par][0], D = S->wd[par][1];
+        __syncwarp();
+        if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
+        backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
+      }
+      u32 stop = 0;
+      if (lane == 0) {
+        stop = meta_term(T.meta[0]) || it >= a.max_iterations;
+        if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
+      }
+      stop = __shfl_sync(kFull, stop, 0);
+      if (!stop) {
+        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
+        if (lane == 0) {
+          s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
+          depth_sum += (unsigned)L.depth;
+          refused += L.refused;
+        }
+      }
+      if (lane == 0) S->stop = stop;
+    }
+    grid.sync();
+    const u32 stop = S->stop;
+    const u64 own = S->own, opp = S->opp;
+    const u32 term = S->term;
+    if (stop) break;
+    int r;
+    if (term) {
+      const int x = __popcll(own), y = __popcll(opp);
+      r = (x > y) - (x < y);
+    } else {
+      r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, s_rays, &plies);
+    }
+    const u32 bw = __popc(__ballot_sync(kFull, r == 1));
+    const u32 bd = __popc(__ballot_sync(kFull, r == 0));
+    if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
+    __syncthreads();
+    if (tid == 0) {
+      const u32 par = it & 1u;
+      atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
+      atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
+    }
+    grid.sync();
+  }
+  const u32 bp = __reduce_add_sync(kFull, plies);
+  if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
+  if (leader && lane == 0 && depth_sum)
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
+  if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
+  if (leader) merge_root(T, 0, unit, it, a.stats, lane);
+}
+
+#else
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
@@ -268,6 +363,8 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
+
+#endif
 
 }  // namespace mcts_dev
 
