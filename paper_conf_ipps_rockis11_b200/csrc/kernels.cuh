@@ -136,31 +136,18 @@ block_search_kernel(TreePool T, SearchArgs a) {
 
 // ---------------------------------------------------------------------------
 // Leaf-parallel UCT: one tree; every thread of the grid
-// plays out from the same leaf each iteration. CTA 0's warp 0 (the leader)
-// owns the tree (select/expand/backprop); all CTAs are co-resident
-// (cooperative launch). One grid barrier per iteration (round 1 used two):
-//   leader: collects iteration it - 1 (waits until all gridDim CTAs have
-//     posted, takes and clears the sums), backpropagates, selects iteration
-//     it's leaf and writes it to S;
-//   grid.sync(): the leaf is published;
-//   every CTA: plays its playouts, reduces them (ballots + shared memory),
-//     adds (1, W, D) to the packed word S->post[it & 1] with one atomic,
-//     then goes straight to the next grid.sync.
-// The parity double-buffer makes the clears safe: slot it & 1 is next posted
-// to two barriers after the leader clears it. Only the leader touches the
-// tree; it polls the posts with relaxed L2 loads, the CTAs read the leaf with
-// .cg loads.
+// plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree
+// (select/expand/backprop); the leaf is published through a small global
+// struct between two cooperative-groups grid barriers per iteration
+// (select -> sync -> simulate + per-CTA ballot reduce + atomics -> sync).
+// All CTAs are co-resident (cooperative launch). (Round 2 measured a
+// one-barrier hand-off — CTAs post their sums with one packed atomic and the
+// leader polls them — 20-27% slower from the opening.)
 // ---------------------------------------------------------------------------
-#ifndef MCTS_LEAF_BARRIERS
-#define MCTS_LEAF_BARRIERS 1  // 2: round 1's two grid barriers per iteration (tuning comparison)
-#endif
-#if MCTS_LEAF_BARRIERS == 2
-struct LeafSync {  // two-barrier variant
+struct LeafSync {
   u64 own, opp;
   u32 term, stop;
   u32 wd[2][2];     // per-iteration-parity wins, draws
-  u32 abort;
-  u32 diag[4];
 };
 
 __global__ void __launch_bounds__(128)
@@ -244,127 +231,6 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
-
-#else
-struct LeafSync {
-  u64 own, opp;
-  u32 term, stop;
-  // Per-iteration-parity posts, one 64-bit word each: CTAs that posted in
-  // bits 0-15, wins in bits 16-39, draws in bits 40-63 (unit <= 65536 < 2^24,
-  // gridDim <= 512 < 2^16). A CTA posts with ONE atomic add, so the leader
-  // reads the count and the sums it covers in one load — no fences, no
-  // acquire (which would invalidate the leader SM's L1, where the hot top of
-  // the tree lives).
-  unsigned long long post[2];
-  u32 abort;        // watchdog: the leader's wait exceeded kLeafWaitNs (diag below)
-  u32 diag[4];      // iteration, count seen, gridDim, 0
-};
-
-// The leader's wait never legitimately exceeds one playout phase
-// (microseconds); past this the kernel aborts (mcts_search reports
-// MCTS_E_CUDA with the diag) instead of hanging the GPU.
-constexpr u64 kLeafWaitNs = 2000000000ULL;
-
-__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
-  unsigned long long v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-
-__global__ void __launch_bounds__(128)
-leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
-  namespace cg = cooperative_groups;
-  cg::grid_group grid = cg::this_grid();
-  __shared__ u32 path[kMaxPath];
-  __shared__ u32 s_slot_used;
-  __shared__ int s_depth;
-  __shared__ u32 s_w[4], s_d[4];
-  __shared__ u64 s_rays[kRayTable];
-  load_rays(s_rays, a.rays);
-
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const bool leader = blockIdx.x == 0 && warp == 0;
-  const u32 unit = a.unit;
-  const u32 G = gridDim.x;
-  const u64 deadline = a.budget_ns ? (*a.t0 + a.budget_ns) : 0ULL;
-  if (blockIdx.x == 0 && tid == 0) {
-    const u64 own = a.root.to_move ? a.root.white : a.root.black;
-    const u64 opp = a.root.to_move ? a.root.black : a.root.white;
-    init_node(T, 0, own, opp, 0xFFu);
-    s_slot_used = 1;
-  }
-  __syncthreads();
-  u32 plies = 0;
-  u32 it = 0;
-  unsigned long long depth_sum = 0;  // leader lane 0
-  unsigned long long refused = 0;    // leader lane 0
-  for (;; ++it) {
-    if (leader) {
-      u32 stop = 0;
-      if (it > 0) {  // collect iteration it - 1 from every CTA, backpropagate
-        const u32 pp = (it - 1u) & 1u;
-        unsigned long long v = 0;
-        if (lane == 0) {
-          const u64 t0 = globaltimer_ns();
-          while (((v = ld_relaxed_u64(&S->post[pp])) & 0xFFFFull) < G) {
-            __nanosleep(20);
-            if (globaltimer_ns() - t0 > kLeafWaitNs) {
-              S->abort = 1u; S->diag[0] = it; S->diag[1] = (u32)(v & 0xFFFFull); S->diag[2] = G; S->diag[3] = 0;
-              break;
-            }
-          }
-          S->post[pp] = 0ull;  // next posted to in iteration it + 1, two barriers later
-        }
-        v = __shfl_sync(kFull, v, 0);
-        const u32 W = (u32)((v >> 16) & 0xFFFFFFull), D = (u32)(v >> 40);
-        backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
-      }
-      if (lane == 0) {
-        stop = S->abort || meta_term(T.meta[0]) || it >= a.max_iterations;
-        if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
-      }
-      stop = __shfl_sync(kFull, stop, 0);
-      if (!stop) {
-        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
-        if (lane == 0) {
-          s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
-          depth_sum += (unsigned)L.depth;
-          refused += L.refused;
-        }
-      }
-      if (lane == 0) S->stop = stop;
-    }
-    grid.sync();
-    const u32 stop = __ldcg(&S->stop);
-    if (stop) break;
-    const u64 own = __ldcg(&S->own), opp = __ldcg(&S->opp);
-    const u32 term = __ldcg(&S->term);
-    int r;
-    if (term) {
-      const int x = __popcll(own), y = __popcll(opp);
-      r = (x > y) - (x < y);
-    } else {
-      r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, s_rays, &plies);
-    }
-    const u32 bw = __popc(__ballot_sync(kFull, r == 1));
-    const u32 bd = __popc(__ballot_sync(kFull, r == 0));
-    if (lane == 0) { s_w[warp] = bw; s_d[warp] = bd; }
-    __syncthreads();
-    if (tid == 0) {  // one atomic: the post count and the sums it covers
-      const unsigned long long w = s_w[0] + s_w[1] + s_w[2] + s_w[3], d = s_d[0] + s_d[1] + s_d[2] + s_d[3];
-      atomicAdd(&S->post[it & 1u], 1ull | (w << 16) | (d << 40));
-    }
-  }
-  if (leader && lane == 0 && S->abort) *a.error = 4;
-  const u32 bp = __reduce_add_sync(kFull, plies);
-  if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
-  if (leader && lane == 0 && depth_sum)
-    atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
-  if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
-  if (leader) merge_root(T, 0, unit, it, a.stats, lane);
-}
-
-#endif
 
 }  // namespace mcts_dev
 

@@ -713,13 +713,6 @@ mcts_status mcts_search(mcts_handle* h, const mcts_position* root, mcts_budget b
   CK(h, cudaMemcpyAsync(&herr, h->d_error, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CK(h, cudaStreamSynchronize(h->stream));
   if (herr == 2) return fail(h, MCTS_E_CUDA, "MCTS_TREE: tree invariant check failed (MCTS_FLAG_CHECK_TREE)");
-  if (herr == 4) {
-    LeafSync ls;
-    CK(h, cudaMemcpy(&ls, h->d_leafsync, sizeof(ls), cudaMemcpyDeviceToHost));
-    return fail(h, MCTS_E_CUDA, "MCTS_LEAF: the leader's wait for the grid timed out (iteration " +
-                                    std::to_string(ls.diag[0]) + ", " + std::to_string(ls.diag[1]) + " of " +
-                                    std::to_string(ls.diag[2]) + " CTAs posted)");  // diag: iteration, posts seen, gridDim
-  }
   if (herr) return fail(h, MCTS_E_CUDA, "search kernel reported an internal error");
   fill_root_stats(hs, out);
   return MCTS_OK;
