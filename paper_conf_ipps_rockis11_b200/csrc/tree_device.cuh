@@ -38,10 +38,11 @@ __device__ __forceinline__ u32 meta_limit(u32 m) { return (m >> 8) & 0xFFu; }
 __device__ __forceinline__ u32 meta_move(u32 m) { return (m >> 16) & 0xFFu; }
 __device__ __forceinline__ bool meta_term(u32 m) { return (m >> 24) != 0u; }
 
-__device__ __forceinline__ void init_node(const TreePool& T, size_t s, u64 own, u64 opp, u32 move) {
+__device__ __forceinline__ u32 init_node(const TreePool& T, size_t s, u64 own, u64 opp, u32 move) {
   const u64 lg = legal_moves(own, opp);
   const bool term = is_terminal(own, opp, lg);
   const u32 limit = term ? 0u : (lg ? (u32)__popcll(lg) : 1u);
+  const u32 meta = (limit << 8) | (move << 16) | ((term ? 1u : 0u) << 24);
   T.own[s] = own;
   T.opp[s] = opp;
   T.legal[s] = lg;
@@ -49,7 +50,8 @@ __device__ __forceinline__ void init_node(const TreePool& T, size_t s, u64 own, 
   T.w[s] = 0;
   T.d[s] = 0;
   T.first[s] = kNoChild;
-  T.meta[s] = (limit << 8) | (move << 16) | ((term ? 1u : 0u) << 24);
+  T.meta[s] = meta;
+  return meta;
 }
 
 // u = w/n + C*sqrt(lnT[k_parent]/n): five IEEE round-to-nearest operations in
@@ -71,29 +73,42 @@ struct LeafInfo {
 // Selection + expansion of one iteration, executed by one full warp.
 // path (shared) receives the node slots root..leaf; *slot_used (shared) is the
 // tree's slot allocator. Returns the leaf (same value in every lane).
+//
+// Latency (round 2): the warp walks the tree through L2, so each level costs
+// its dependent round trips. A level's lanes load their children's (w, k)
+// for UCB together with the children's control values (meta, first), and the
+// winner's are broadcast from its lane, so descending one level is ONE round
+// trip (plus lnT[k], whose address is known as soon as the parent is chosen)
+// instead of five (meta, first, k, lnT, children). Only this warp writes the
+// tree (block and leaf schemes), so the values read are the current ones.
 __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base, u32* path,
                                                   u32* slot_used, const double* __restrict__ lnT,
                                                   u32 unit, double C, int lane) {
   u32 v = 0;
   int depth = 0;
   if (lane == 0) path[0] = 0;
-  // Control values (meta, first child, parent count) are read by lane 0 and
-  // broadcast, so every lane takes the same path through the loop whatever the
-  // memory system returns to each lane's own load (a leaf kernel whose leader
-  // lanes loaded them individually diverged and deadlocked).
-  u32 meta = __shfl_sync(kFull, T.meta[base], 0);
+  // Control values (meta, first child, count) of the current node are read by
+  // one lane and broadcast, so every lane takes the same path through the
+  // loop whatever the memory system returns to each lane's own load (a leaf
+  // kernel whose leader lanes loaded them individually diverged and
+  // deadlocked).
+  u32 meta = 0, first = 0, kv = 0;
+  if (lane == 0) { meta = T.meta[base]; first = T.first[base]; kv = T.k[base]; }
+  meta = __shfl_sync(kFull, meta, 0);
+  first = __shfl_sync(kFull, first, 0);
+  kv = __shfl_sync(kFull, kv, 0);
   // Selection (L157-L178): descend while the node is non-terminal and fully expanded.
   // (depth bound: a game has < 128 plies incl. passes; never reached)
   while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta) && depth < kMaxPath - 2) {
     const u32 nch = meta_nchild(meta);
-    const u32 first = __shfl_sync(kFull, T.first[base + v], 0);
-    const double lnp = lnT[__shfl_sync(kFull, T.k[base + v], 0)];
+    const double lnp = lnT[kv];
     double best_u = -__longlong_as_double(0x7FF0000000000000LL);  // -inf
-    u32 best_i = kNoChild;
+    u32 best_i = kNoChild, best_meta = 0, best_first = 0, best_k = 0;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
       const size_t c = base + first + i;
-      const double u = ucb_value(T.w[c], T.k[c], unit, lnp, C);
-      if (u > best_u) { best_u = u; best_i = i; }
+      const u32 wc = T.w[c], kc = T.k[c], mc = T.meta[c], fc = T.first[c];
+      const double u = ucb_value(wc, kc, unit, lnp, C);
+      if (u > best_u) { best_u = u; best_i = i; best_meta = mc; best_first = fc; best_k = kc; }
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
@@ -101,53 +116,67 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
       const u32 oi = __shfl_xor_sync(kFull, best_i, off);
       if (ou > best_u || (ou == best_u && oi < best_i)) { best_u = ou; best_i = oi; }
     }
+    // child best_i was scored by lane best_i mod 32, whose own best it is
+    const int src = (int)(best_i & 31u);
     v = first + best_i;
+    meta = __shfl_sync(kFull, best_meta, src);
+    first = __shfl_sync(kFull, best_first, src);
+    kv = __shfl_sync(kFull, best_k, src);
     ++depth;
     if (lane == 0) path[depth] = v;
-    meta = __shfl_sync(kFull, T.meta[base + v], 0);
   }
   // Expansion (L179-L182): the lowest-index untried move, or the pass child.
+  // Lane 0 reads v's board once; the leaf it returns is v or the new child,
+  // from registers.
   LeafInfo L;
   L.refused = 0;
-  if (!meta_term(meta)) {
-    u32 c = kNoChild;
-    if (lane == 0) {
+  u32 c = kNoChild;
+  u64 own = 0, opp = 0;
+  u32 term = meta_term(meta) ? 1u : 0u;
+  if (lane == 0) {
+    own = T.own[base + v];
+    opp = T.opp[base + v];
+    const u64 lg = T.legal[base + v];
+    if (!term) {
       const u32 nch = meta_nchild(meta), limit = meta_limit(meta);
-      u32 first = T.first[base + v];
+      u32 f0 = first;
       if (nch == 0u) {
         if (*slot_used + limit <= T.slot_cap) {
-          first = *slot_used;
+          f0 = *slot_used;
           *slot_used += limit;
-          T.first[base + v] = first;
+          T.first[base + v] = f0;
         } else {
-          first = kNoChild;  // pool full (time mode): simulate from v itself
+          f0 = kNoChild;  // pool full (time mode): simulate from v itself
           L.refused = 1;
         }
       }
-      if (first != kNoChild) {
-        const u64 own = T.own[base + v], opp = T.opp[base + v], lg = T.legal[base + v];
-        c = first + nch;
+      if (f0 != kNoChild) {
+        c = f0 + nch;
+        u64 cown, copp;
+        u32 mv;
         if (lg == 0ULL) {
-          init_node(T, base + c, opp, own, 64u);  // pass: same discs, turn swaps
+          cown = opp; copp = own; mv = 64u;  // pass: same discs, turn swaps
         } else {
           const int sq = kth_set_bit(lg, nch);
           const u64 f = flips(sq, own, opp);
-          init_node(T, base + c, opp & ~f, own | f | (1ULL << sq), (u32)sq);
+          cown = opp & ~f; copp = own | f | (1ULL << sq); mv = (u32)sq;
         }
+        term = meta_term(init_node(T, base + c, cown, copp, mv)) ? 1u : 0u;
         T.meta[base + v] = meta + 1u;  // ++nchild
         path[depth + 1] = c;
+        own = cown; opp = copp;
       }
     }
-    c = __shfl_sync(kFull, c, 0);
-    __syncwarp();
-    if (c != kNoChild) {
-      v = c;
-      ++depth;
-    }
   }
-  L.own = T.own[base + v];
-  L.opp = T.opp[base + v];
-  L.term = meta_term(T.meta[base + v]) ? 1u : 0u;
+  c = __shfl_sync(kFull, c, 0);
+  __syncwarp();
+  if (c != kNoChild) {
+    v = c;
+    ++depth;
+  }
+  L.own = __shfl_sync(kFull, own, 0);
+  L.opp = __shfl_sync(kFull, opp, 0);
+  L.term = __shfl_sync(kFull, term, 0);
   L.depth = depth;
   return L;
 }
