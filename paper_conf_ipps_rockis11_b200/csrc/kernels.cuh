@@ -51,7 +51,7 @@ struct SearchArgs {
 template <int MAX_THREADS, int MIN_BLOCKS>
 __global__ void __launch_bounds__(MAX_THREADS, MIN_BLOCKS)
 block_search_kernel(TreePool T, SearchArgs a) {
-  __shared__ u32 path[kMaxPath];
+  __shared__ PathCache pc;
   __shared__ u64 s_own, s_opp;
   __shared__ u32 s_term, s_stop, s_slot_used;
   __shared__ u32 s_w[32], s_d[32];
@@ -70,7 +70,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
   if (tid == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
     const u64 opp = a.root.to_move ? a.root.black : a.root.white;
-    init_node(T, base, own, opp, 0xFFu);
+    init_root(T, base, own, opp, &pc);
     s_slot_used = 1;
   }
   __syncthreads();
@@ -79,7 +79,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
   u32 it = 0;
   unsigned long long depth_sum = 0;  // lane 0 of warp 0: sum of leaf depths (Fig. 8 "Depth")
   unsigned long long refused = 0;    // lane 0 of warp 0: expansions refused by a full pool
-  if (!meta_term(T.meta[base])) {
+  if (!meta_term(pc.root_meta)) {
     for (;; ++it) {
       if (warp == 0) {
         u32 stop = 0;
@@ -89,7 +89,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
         }
         stop = __shfl_sync(kFull, stop, 0);
         if (!stop) {
-          const LeafInfo L = select_expand(T, base, path, &s_slot_used, a.lnT, unit, a.C, lane);
+          const LeafInfo L = select_expand(T, base, &pc, &s_slot_used, a.lnT, unit, a.C, lane, s_rays);
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth;
             depth_sum += (unsigned)L.depth;
@@ -116,7 +116,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
         u32 D = lane < nwarps ? s_d[lane] : 0u;
         W = __reduce_add_sync(kFull, W);
         D = __reduce_add_sync(kFull, D);
-        backprop(T, base, path, s_depth, W, D, unit - W - D, lane);
+        backprop(T, base, &pc, s_depth, W, D, unit - W - D, lane);
       }
     }
   }
@@ -129,7 +129,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
     for (int off = 16; off > 0; off >>= 1) P += __shfl_xor_sync(kFull, P, off);
     if (lane == 0 && P) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, P);
     if (lane == 0 && depth_sum) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
-    if (lane == 0 && !meta_term(T.meta[base])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
+    if (lane == 0 && !meta_term(pc.root_meta)) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
     merge_root(T, base, unit, it, a.stats, lane);
   }
 }
@@ -144,6 +144,13 @@ block_search_kernel(TreePool T, SearchArgs a) {
 // one-barrier hand-off — CTAs post their sums with one packed atomic and the
 // leader polls them — 20-27% slower from the opening.)
 // ---------------------------------------------------------------------------
+// Tooling only (tools/leaf_compare.py variants): 1 = the leaf kernel skips the
+// playouts (every result a draw), so its iteration time is the serial part
+// alone (barriers, backprop, selection, expansion). Never set in a product build.
+#ifndef MCTS_LEAF_PROBE
+#define MCTS_LEAF_PROBE 0
+#endif
+
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
@@ -154,7 +161,7 @@ __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   namespace cg = cooperative_groups;
   cg::grid_group grid = cg::this_grid();
-  __shared__ u32 path[kMaxPath];
+  __shared__ PathCache pc;
   __shared__ u32 s_slot_used;
   __shared__ int s_depth;
   __shared__ u32 s_w[4], s_d[4];
@@ -168,7 +175,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (blockIdx.x == 0 && tid == 0) {
     const u64 own = a.root.to_move ? a.root.white : a.root.black;
     const u64 opp = a.root.to_move ? a.root.black : a.root.white;
-    init_node(T, 0, own, opp, 0xFFu);
+    init_root(T, 0, own, opp, &pc);
     s_slot_used = 1;
   }
   __syncthreads();
@@ -183,16 +190,16 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
         const u32 W = S->wd[par][0], D = S->wd[par][1];
         __syncwarp();
         if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
-        backprop(T, 0, path, s_depth, W, D, unit - W - D, lane);
+        backprop(T, 0, &pc, s_depth, W, D, unit - W - D, lane);
       }
       u32 stop = 0;
       if (lane == 0) {
-        stop = meta_term(T.meta[0]) || it >= a.max_iterations;
+        stop = meta_term(pc.root_meta) || it >= a.max_iterations;
         if (!stop && a.budget_ns) stop = globaltimer_ns() >= deadline;
       }
       stop = __shfl_sync(kFull, stop, 0);
       if (!stop) {
-        const LeafInfo L = select_expand(T, 0, path, &s_slot_used, a.lnT, unit, a.C, lane);
+        const LeafInfo L = select_expand(T, 0, &pc, &s_slot_used, a.lnT, unit, a.C, lane, s_rays);
         if (lane == 0) {
           s_depth = L.depth; S->own = L.own; S->opp = L.opp; S->term = L.term;
           depth_sum += (unsigned)L.depth;
@@ -211,7 +218,11 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
       const int x = __popcll(own), y = __popcll(opp);
       r = (x > y) - (x < y);
     } else {
+#if MCTS_LEAF_PROBE
+      r = 0;
+#else
       r = playout(own, opp, a.key, a.tree_id_base, it, blockIdx.x * blockDim.x + tid, s_rays, &plies);
+#endif
     }
     const u32 bw = __popc(__ballot_sync(kFull, r == 1));
     const u32 bd = __popc(__ballot_sync(kFull, r == 0));
@@ -228,7 +239,7 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);
   if (leader && lane == 0 && depth_sum)
     atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 198, depth_sum);
-  if (leader && lane == 0 && !meta_term(T.meta[0])) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
+  if (leader && lane == 0 && !meta_term(pc.root_meta)) merge_pool(a.stats, refused, s_slot_used, T.slot_cap);
   if (leader) merge_root(T, 0, unit, it, a.stats, lane);
 }
 

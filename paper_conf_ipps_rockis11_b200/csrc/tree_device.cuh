@@ -38,9 +38,21 @@ __device__ __forceinline__ u32 meta_limit(u32 m) { return (m >> 8) & 0xFFu; }
 __device__ __forceinline__ u32 meta_move(u32 m) { return (m >> 16) & 0xFFu; }
 __device__ __forceinline__ bool meta_term(u32 m) { return (m >> 24) != 0u; }
 
-__device__ __forceinline__ u32 init_node(const TreePool& T, size_t s, u64 own, u64 opp, u32 move) {
-  const u64 lg = legal_moves(own, opp);
-  const bool term = is_terminal(own, opp, lg);
+// Create node s (one thread). With `hot` the hot-loop move generator
+// (legal_moves_hot, pinned by the device perft) replaces the plain one.
+// Returns the meta word; *lg_out (optional) receives the legal moves.
+__device__ __forceinline__ u32 init_node(const TreePool& T, size_t s, u64 own, u64 opp, u32 move,
+                                         bool hot = false, u64* lg_out = nullptr) {
+  u64 lg;
+  bool term;
+  if (hot) {
+    const u64 ro = __brevll(own), rp = __brevll(opp);
+    lg = legal_moves_hot(own, opp, ro, rp);
+    term = lg == 0ULL && legal_moves_hot(opp, own, rp, ro) == 0ULL;
+  } else {
+    lg = legal_moves(own, opp);
+    term = is_terminal(own, opp, lg);
+  }
   const u32 limit = term ? 0u : (lg ? (u32)__popcll(lg) : 1u);
   const u32 meta = (limit << 8) | (move << 16) | ((term ? 1u : 0u) << 24);
   T.own[s] = own;
@@ -51,6 +63,32 @@ __device__ __forceinline__ u32 init_node(const TreePool& T, size_t s, u64 own, u
   T.d[s] = 0;
   T.first[s] = kNoChild;
   T.meta[s] = meta;
+  if (lg_out) *lg_out = lg;
+  return meta;
+}
+
+// The owning warp's view of its current path (shared memory; block and leaf
+// schemes, where one warp is the tree's only reader and writer): the node
+// slots root..leaf with the (k, w, d) it last read or wrote for each, and the
+// root's board and control values. Selection fills it, backpropagation
+// writes the updated statistics from it without reading the tree again, and
+// the root (position 0) stays current across iterations, so an iteration
+// reads the tree only at the levels it descends.
+struct PathCache {
+  u32 node[kMaxPath];
+  u32 k[kMaxPath], w[kMaxPath], d[kMaxPath];
+  u64 root_own, root_opp, root_legal;
+  u32 root_meta, root_first;
+};
+
+// Create the root (one thread) and its cache entry.
+__device__ __forceinline__ u32 init_root(const TreePool& T, size_t base, u64 own, u64 opp, PathCache* pc) {
+  u64 lg;
+  const u32 meta = init_node(T, base, own, opp, 0xFFu, true, &lg);
+  pc->node[0] = 0;
+  pc->k[0] = 0; pc->w[0] = 0; pc->d[0] = 0;
+  pc->root_own = own; pc->root_opp = opp; pc->root_legal = lg;
+  pc->root_meta = meta; pc->root_first = kNoChild;
   return meta;
 }
 
@@ -70,45 +108,52 @@ struct LeafInfo {
   int depth;
 };
 
-// Selection + expansion of one iteration, executed by one full warp.
-// path (shared) receives the node slots root..leaf; *slot_used (shared) is the
-// tree's slot allocator. Returns the leaf (same value in every lane).
+// Selection + expansion of one iteration, executed by one full warp that
+// owns the tree. pc (shared) receives the path root..leaf and its
+// statistics; *slot_used (shared) is the tree's slot allocator; rays is the
+// CTA's shared ray table (flips_loop). Returns the leaf (same value in every
+// lane).
 //
 // Latency (round 2): the warp walks the tree through L2, so each level costs
-// its dependent round trips. A level's lanes load their children's (w, k)
-// for UCB together with the children's control values (meta, first), and the
-// winner's are broadcast from its lane, so descending one level is ONE round
-// trip (plus lnT[k], whose address is known as soon as the parent is chosen)
-// instead of five (meta, first, k, lnT, children). Only this warp writes the
-// tree (block and leaf schemes), so the values read are the current ones.
-__device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base, u32* path,
+// its dependent round trips. A level's lanes load their children's UCB
+// statistics (w, k) together with everything the next step needs (d, meta,
+// first, board, legal moves), and the winner's values are broadcast from its
+// lane: descending one level is ONE round trip (lnT[k] is issued alongside),
+// the root comes from the cache, and the expansion needs no read at all —
+// instead of the five dependent reads per level, a root read and a board read
+// of round 1.
+__device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base, PathCache* pc,
                                                   u32* slot_used, const double* __restrict__ lnT,
-                                                  u32 unit, double C, int lane) {
+                                                  u32 unit, double C, int lane,
+                                                  const u64* __restrict__ rays) {
   u32 v = 0;
   int depth = 0;
-  if (lane == 0) path[0] = 0;
-  // Control values (meta, first child, count) of the current node are read by
-  // one lane and broadcast, so every lane takes the same path through the
-  // loop whatever the memory system returns to each lane's own load (a leaf
-  // kernel whose leader lanes loaded them individually diverged and
-  // deadlocked).
+  // Control values are read by one lane and broadcast, so every lane takes the
+  // same path through the loop (a leaf kernel whose leader lanes loaded them
+  // individually diverged and deadlocked).
   u32 meta = 0, first = 0, kv = 0;
-  if (lane == 0) { meta = T.meta[base]; first = T.first[base]; kv = T.k[base]; }
+  if (lane == 0) { meta = pc->root_meta; first = pc->root_first; kv = pc->k[0]; }
   meta = __shfl_sync(kFull, meta, 0);
   first = __shfl_sync(kFull, first, 0);
   kv = __shfl_sync(kFull, kv, 0);
+  u64 own = pc->root_own, opp = pc->root_opp, lg = pc->root_legal;  // used by lane 0 only
   // Selection (L157-L178): descend while the node is non-terminal and fully expanded.
   // (depth bound: a game has < 128 plies incl. passes; never reached)
   while (!meta_term(meta) && meta_nchild(meta) >= meta_limit(meta) && depth < kMaxPath - 2) {
     const u32 nch = meta_nchild(meta);
     const double lnp = lnT[kv];
     double best_u = -__longlong_as_double(0x7FF0000000000000LL);  // -inf
-    u32 best_i = kNoChild, best_meta = 0, best_first = 0, best_k = 0;
+    u32 best_i = kNoChild, bm = 0, bf = 0, bk = 0, bw = 0, bd = 0;
+    u64 bo = 0, bp = 0, bl = 0;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
       const size_t c = base + first + i;
-      const u32 wc = T.w[c], kc = T.k[c], mc = T.meta[c], fc = T.first[c];
+      const u32 wc = T.w[c], kc = T.k[c], dc = T.d[c], mc = T.meta[c], fc = T.first[c];
+      const u64 oc = T.own[c], pc_ = T.opp[c], lc = T.legal[c];
       const double u = ucb_value(wc, kc, unit, lnp, C);
-      if (u > best_u) { best_u = u; best_i = i; best_meta = mc; best_first = fc; best_k = kc; }
+      if (u > best_u) {
+        best_u = u; best_i = i;
+        bm = mc; bf = fc; bk = kc; bw = wc; bd = dc; bo = oc; bp = pc_; bl = lc;
+      }
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
@@ -119,61 +164,57 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
     // child best_i was scored by lane best_i mod 32, whose own best it is
     const int src = (int)(best_i & 31u);
     v = first + best_i;
-    meta = __shfl_sync(kFull, best_meta, src);
-    first = __shfl_sync(kFull, best_first, src);
-    kv = __shfl_sync(kFull, best_k, src);
+    meta = __shfl_sync(kFull, bm, src);
+    first = __shfl_sync(kFull, bf, src);
+    kv = __shfl_sync(kFull, bk, src);
+    const u32 wv = __shfl_sync(kFull, bw, src), dv = __shfl_sync(kFull, bd, src);
+    own = __shfl_sync(kFull, bo, src);
+    opp = __shfl_sync(kFull, bp, src);
+    lg = __shfl_sync(kFull, bl, src);
     ++depth;
-    if (lane == 0) path[depth] = v;
+    if (lane == 0) { pc->node[depth] = v; pc->k[depth] = kv; pc->w[depth] = wv; pc->d[depth] = dv; }
   }
-  // Expansion (L179-L182): the lowest-index untried move, or the pass child.
-  // Lane 0 reads v's board once; the leaf it returns is v or the new child,
-  // from registers.
+  // Expansion (L179-L182), lane 0: the lowest-index untried move, or the pass
+  // child. The leaf returned is v or the new child, from registers.
   LeafInfo L;
   L.refused = 0;
   u32 c = kNoChild;
-  u64 own = 0, opp = 0;
   u32 term = meta_term(meta) ? 1u : 0u;
-  if (lane == 0) {
-    own = T.own[base + v];
-    opp = T.opp[base + v];
-    const u64 lg = T.legal[base + v];
-    if (!term) {
-      const u32 nch = meta_nchild(meta), limit = meta_limit(meta);
-      u32 f0 = first;
-      if (nch == 0u) {
-        if (*slot_used + limit <= T.slot_cap) {
-          f0 = *slot_used;
-          *slot_used += limit;
-          T.first[base + v] = f0;
-        } else {
-          f0 = kNoChild;  // pool full (time mode): simulate from v itself
-          L.refused = 1;
-        }
+  if (lane == 0 && !term) {
+    const u32 nch = meta_nchild(meta), limit = meta_limit(meta);
+    u32 f0 = first;
+    if (nch == 0u) {
+      if (*slot_used + limit <= T.slot_cap) {
+        f0 = *slot_used;
+        *slot_used += limit;
+        T.first[base + v] = f0;
+      } else {
+        f0 = kNoChild;  // pool full (time mode): simulate from v itself
+        L.refused = 1;
       }
-      if (f0 != kNoChild) {
-        c = f0 + nch;
-        u64 cown, copp;
-        u32 mv;
-        if (lg == 0ULL) {
-          cown = opp; copp = own; mv = 64u;  // pass: same discs, turn swaps
-        } else {
-          const int sq = kth_set_bit(lg, nch);
-          const u64 f = flips(sq, own, opp);
-          cown = opp & ~f; copp = own | f | (1ULL << sq); mv = (u32)sq;
-        }
-        term = meta_term(init_node(T, base + c, cown, copp, mv)) ? 1u : 0u;
-        T.meta[base + v] = meta + 1u;  // ++nchild
-        path[depth + 1] = c;
-        own = cown; opp = copp;
+    }
+    if (f0 != kNoChild) {
+      c = f0 + nch;
+      u64 cown, copp;
+      u32 mv;
+      if (lg == 0ULL) {
+        cown = opp; copp = own; mv = 64u;  // pass: same discs, turn swaps
+      } else {
+        const int sq = kth_set_bit(lg, nch);
+        const u64 f = flips_loop(sq, own, opp, __brevll(own), __brevll(opp), rays);
+        cown = opp & ~f; copp = own | f | (1ULL << sq); mv = (u32)sq;
       }
+      term = meta_term(init_node(T, base + c, cown, copp, mv, true)) ? 1u : 0u;
+      T.meta[base + v] = meta + 1u;  // ++nchild
+      if (depth == 0) { pc->root_meta = meta + 1u; pc->root_first = f0; }
+      pc->node[depth + 1] = c;
+      pc->k[depth + 1] = 0; pc->w[depth + 1] = 0; pc->d[depth + 1] = 0;
+      own = cown; opp = copp;
     }
   }
   c = __shfl_sync(kFull, c, 0);
   __syncwarp();
-  if (c != kNoChild) {
-    v = c;
-    ++depth;
-  }
+  if (c != kNoChild) ++depth;
   L.own = __shfl_sync(kFull, own, 0);
   L.opp = __shfl_sync(kFull, opp, 0);
   L.term = __shfl_sync(kFull, term, 0);
@@ -181,17 +222,21 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
   return L;
 }
 
-// Backpropagation (L196-L199) by one warp, lanes over path positions (distinct
-// nodes). W/D/Lo are the leaf batch's wins/draws/losses for the leaf's side to
-// move; the leaf's mover collects Lo, its parent W, alternating to the root.
-__device__ __forceinline__ void backprop(const TreePool& T, size_t base, const u32* path, int depth,
+// Backpropagation (L196-L199) by the owning warp, lanes over path positions
+// (distinct nodes), from the cached statistics (stores only). W/D/Lo are the
+// leaf batch's wins/draws/losses for the leaf's side to move; the leaf's mover
+// collects Lo, its parent W, alternating to the root. The root's cache entry
+// is kept current.
+__device__ __forceinline__ void backprop(const TreePool& T, size_t base, PathCache* pc, int depth,
                                          u32 W, u32 D, u32 Lo, int lane) {
   for (int p = lane; p <= depth; p += 32) {
-    const size_t s = base + path[p];
+    const size_t s = base + pc->node[p];
     const int lvl = depth - p;
-    T.k[s] += 1u;
-    T.w[s] += (lvl & 1) ? W : Lo;
-    T.d[s] += D;
+    const u32 k = pc->k[p] + 1u, w = pc->w[p] + ((lvl & 1) ? W : Lo), d = pc->d[p] + D;
+    T.k[s] = k;
+    T.w[s] = w;
+    T.d[s] = d;
+    if (p == 0) { pc->k[0] = k; pc->w[0] = w; pc->d[0] = d; }
   }
   __syncwarp();
 }

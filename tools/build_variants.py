@@ -30,6 +30,7 @@ VARIANTS = {
     "t128m10": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=10"],
     "t128m11": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=11"],
     "t64m20": ["MCTS_PLAYOUT_THREADS=64", "MCTS_PLAYOUT_MINB=20"],
+    "leafprobe": ["MCTS_LEAF_PROBE=1"],
 }
 
 if __name__ == "__main__":
