@@ -37,12 +37,15 @@ struct mcts_handle {
   cudaStream_t stream = nullptr;  // for the synchronous entry points
   std::string last_error;
 
-  // playout staging
+  // playout staging. d_wdl (mcts_playouts) is one region zeroed by one memset:
+  // [u32 work counter, u32 pad, u64 plies, n x WdlOut]; h_pin_plies is the
+  // pinned landing slot of its ply count.
   DevPosition* d_leaves = nullptr;
   size_t leaves_cap = 0;
-  WdlOut* d_wdl = nullptr;
+  void* d_wdl = nullptr;
   size_t wdl_cap = 0;
   unsigned long long* d_plies = nullptr;
+  unsigned long long* h_pin_plies = nullptr;
 
   // trees
   void* pool_mem = nullptr;
@@ -570,6 +573,7 @@ mcts_status mcts_create(const mcts_position* position, const mcts_params* params
   if (e == cudaSuccess) e = cudaMalloc(&h->d_treesync, sizeof(TreeSync));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_rays, kRayTable * sizeof(u64));
   if (e == cudaSuccess) e = cudaMalloc(&h->d_work, kWorkSlots * sizeof(u32));
+  if (e == cudaSuccess) e = cudaHostAlloc(&h->h_pin_plies, sizeof(unsigned long long), cudaHostAllocDefault);
   if (e == cudaSuccess) {
     rays_init_kernel<<<1, 256, 0, h->stream>>>(h->d_rays);
     e = cudaGetLastError();
@@ -607,10 +611,30 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_work);
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
+  if (h->h_pin_plies) cudaFreeHost(h->h_pin_plies);
   if (h->step_event) cudaEventDestroy(h->step_event);
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
+
+namespace {
+
+// The playout kernel on a zeroed output and a zeroed work counter (the
+// callers own the memsets).
+mcts_status launch_playouts(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
+                            uint32_t n_per_leaf, uint64_t seed, uint32_t c0_base, uint32_t c1,
+                            mcts_wdl* d_out, uint64_t* d_plies, u32* work, cudaStream_t s) {
+  const uint64_t total = (uint64_t)n_leaves * n_per_leaf;
+  const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
+  const unsigned blocks = (unsigned)(need < (uint64_t)h->playout_ctas ? need : (uint64_t)h->playout_ctas);
+  playouts_kernel<<<blocks, kPlayoutThreads, 0, s>>>(
+      (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), c0_base, c1, (WdlOut*)d_out,
+      (unsigned long long*)d_plies, h->d_rays, work);
+  CK(h, cudaGetLastError());
+  return MCTS_OK;
+}
+
+}  // namespace
 
 mcts_status mcts_playouts_ex_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
                                    uint32_t n_per_leaf, uint64_t seed, uint32_t c0_base, uint32_t c1,
@@ -625,16 +649,10 @@ mcts_status mcts_playouts_ex_async(mcts_handle* h, const mcts_position* d_leaves
   const uint64_t total = (uint64_t)n_leaves * n_per_leaf;
   if (total == 0) return MCTS_OK;
   if ((total + 31) / 32 > 0xFFFFFFF0ull) return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large (>= 2^37 playouts)");
-  const uint64_t need = (total + kPlayoutThreads - 1) / kPlayoutThreads;
-  const unsigned blocks = (unsigned)(need < (uint64_t)h->playout_ctas ? need : (uint64_t)h->playout_ctas);
   // a fresh counter per launch, so launches on different streams do not share one
   u32* work = h->d_work + (h->work_slot++ % kWorkSlots);
   CK(h, cudaMemsetAsync(work, 0, sizeof(u32), s));
-  playouts_kernel<<<blocks, kPlayoutThreads, 0, s>>>(
-      (const DevPosition*)d_leaves, n_leaves, n_per_leaf, key_of(seed), c0_base, c1, (WdlOut*)d_out,
-      (unsigned long long*)d_plies, h->d_rays, work);
-  CK(h, cudaGetLastError());
-  return MCTS_OK;
+  return launch_playouts(h, d_leaves, n_leaves, n_per_leaf, seed, c0_base, c1, d_out, d_plies, work, s);
 }
 
 mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, uint32_t n_leaves,
@@ -644,6 +662,11 @@ mcts_status mcts_playouts_async(mcts_handle* h, const mcts_position* d_leaves, u
                                 stream);
 }
 
+// Host buffers: five stream operations per call — one memset zeroes the work
+// counter, the ply count and the W/D/L counts together (one region), the
+// leaves go up, the kernel runs, the counts come down into the caller's
+// buffer and the ply count into a pinned slot (a pageable 8-byte copy would be
+// staged by the driver).
 mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
                           uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts, uint64_t* out_plies) {
   if (!h) return MCTS_E_INVALID_ARGUMENT;
@@ -665,21 +688,24 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
   st = ensure(h, &p, &h->leaves_cap, (size_t)n_leaves * sizeof(DevPosition));
   if (st) return st;
   h->d_leaves = (DevPosition*)p;
-  p = h->d_wdl;
-  st = ensure(h, &p, &h->wdl_cap, (size_t)n_leaves * sizeof(WdlOut));
+  constexpr size_t kHead = 16;  // u32 work, u32 pad, u64 plies
+  const size_t region = kHead + (size_t)n_leaves * sizeof(WdlOut);
+  st = ensure(h, &h->d_wdl, &h->wdl_cap, region);
   if (st) return st;
-  h->d_wdl = (WdlOut*)p;
+  char* base = (char*)h->d_wdl;
+  u32* work = (u32*)base;
+  uint64_t* d_plies = (uint64_t*)(base + 8);
+  mcts_wdl* d_out = (mcts_wdl*)(base + kHead);
   cudaStream_t s = h->stream;
-  CK(h, cudaMemsetAsync(h->d_plies, 0, sizeof(unsigned long long), s));
+  CK(h, cudaMemsetAsync(base, 0, region, s));
   CK(h, cudaMemcpyAsync(h->d_leaves, leaf_batch, (size_t)n_leaves * sizeof(DevPosition), cudaMemcpyHostToDevice, s));
-  st = mcts_playouts_async(h, (const mcts_position*)h->d_leaves, n_leaves, n_per_leaf, seed, 0,
-                           (mcts_wdl*)h->d_wdl, (uint64_t*)h->d_plies, s);
+  st = launch_playouts(h, (const mcts_position*)h->d_leaves, n_leaves, n_per_leaf, seed, 0u, 0u, d_out,
+                       d_plies, work, s);
   if (st) return st;
-  CK(h, cudaMemcpyAsync(out_counts, h->d_wdl, (size_t)n_leaves * sizeof(WdlOut), cudaMemcpyDeviceToHost, s));
-  unsigned long long plies = 0;
-  CK(h, cudaMemcpyAsync(&plies, h->d_plies, sizeof(plies), cudaMemcpyDeviceToHost, s));
+  CK(h, cudaMemcpyAsync(out_counts, d_out, (size_t)n_leaves * sizeof(WdlOut), cudaMemcpyDeviceToHost, s));
+  CK(h, cudaMemcpyAsync(h->h_pin_plies, d_plies, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   CK(h, cudaStreamSynchronize(s));
-  if (out_plies) *out_plies = plies;
+  if (out_plies) *out_plies = *h->h_pin_plies;
   return MCTS_OK;
 }
 
@@ -811,10 +837,8 @@ mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_b
   st = ensure(h, &p, &h->leaves_cap, (size_t)n_trees * sizeof(DevPosition));
   if (st) return st;
   h->d_leaves = (DevPosition*)p;
-  p = h->d_wdl;
-  st = ensure(h, &p, &h->wdl_cap, (size_t)n_trees * sizeof(WdlOut));
+  st = ensure(h, &h->d_wdl, &h->wdl_cap, (size_t)n_trees * sizeof(WdlOut));
   if (st) return st;
-  h->d_wdl = (WdlOut*)p;
   CK(h, cudaMemsetAsync(h->d_plies, 0, sizeof(unsigned long long), h->stream));
 
   HostedGpu g{h, seed, threads_per_tree, (mcts_position*)h->d_leaves, (mcts_wdl*)h->d_wdl, h->d_plies, cudaSuccess};

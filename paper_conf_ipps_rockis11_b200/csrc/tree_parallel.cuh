@@ -125,9 +125,20 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
   u32 refused = 0;
   for (;;) {
     if (meta_term(meta) || depth >= kMaxPath - 2) break;
-    if (first == kNoChild) {  // pool full when v was created (or a racing read): simulate from v
-      refused = 1;
-      break;
+    if (first == kNoChild) {
+      // Either v's child block was refused when v was created (pool full, R12)
+      // or the batch read of v's fields raced its publication (meta seen,
+      // first still the cleared value). Lane 0 re-reads first after a fence,
+      // so only a real refusal is counted; either way v is simulated in place.
+      if (lane == 0) {
+        __threadfence();
+        first = ld_acq(&T.first[v]);
+      }
+      first = __shfl_sync(kFull, first, 0);
+      if (first == kNoChild) {
+        refused = 1;
+        break;
+      }
     }
     // Expansion: claim the lowest-index untried move (one CAS on the counter).
     if (meta_nchild(meta) < meta_limit(meta)) {
