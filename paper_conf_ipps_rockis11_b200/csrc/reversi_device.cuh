@@ -580,4 +580,102 @@ __device__ __forceinline__ int playout(u64 me, u64 op, uint2 key, u32 c0, u32 c1
   return (a > b) - (a < b);
 }
 
+
+// ---------------------------------------------------------------------------
+// Two playouts per thread (MCTS_PAIR tuning variant): playouts X
+// and Y advance in lock step, one ply each per half-step, so the compiler can
+// interleave their independent instruction streams. Each half-step is one
+// branch-free block (movegen, pick, flips and a board update masked by "has a
+// move", as IMADs by 0/1) preceded by the rare Philox refills and followed by
+// the pass / game-end bookkeeping; a finished playout keeps computing on an
+// empty move mask and changes nothing. Same RNG words, same moves, same
+// results as playout() for each of the two.
+// ---------------------------------------------------------------------------
+struct PairSide {
+  u32 n, empties, c0, c2;
+  uint4 buf;
+  bool fresh, passed, done;
+};
+
+__device__ __forceinline__ void pair_init(PairSide& X, u64 me, u64 op, u32 c0, u32 c2, bool act) {
+  X.n = 0;
+  X.empties = 64u - (u32)__popcll(me | op);
+  X.c0 = c0;
+  X.c2 = c2;
+  X.buf = make_uint4(0, 0, 0, 0);
+  X.fresh = false;
+  X.passed = false;
+  X.done = !act || X.empties == 0u;
+}
+
+__device__ __forceinline__ void pair_refill(PairSide& X, uint2 key, u32 c1) {
+  if (!X.done && (X.n & 3u) == 0u && !X.fresh) {
+    X.buf = philox4x32_10(make_uint4(X.c0, c1, X.c2, X.n >> 2), key);
+    X.fresh = true;
+  }
+}
+
+// The branch-free part of one decision for the side owning P: returns whether
+// a move was played (P, O updated).
+__device__ __forceinline__ bool pair_ply(u64& P, u64& O, const PairSide& X, const u64* __restrict__ rays) {
+  const u64 rP = __brevll(P), rO = __brevll(O);
+  u64 moves = legal_moves_hot(P, O, rP, rO);
+  moves = X.done ? 0ULL : moves;
+  const bool has = ((u32)moves | (u32)(moves >> 32)) != 0u;
+  const u32 k = __umulhi(X.buf.x, (u32)__popcll(moves));
+  bool hx;
+  const int sq = kth_set_bit_lut(moves, k, reinterpret_cast<const unsigned char*>(rays + 512), &hx);
+  const u64 f = flips_hot_xy(sq, P, O, rP, rO, rays, hx);
+  const u32 h = has ? 1u : 0u;
+  const u64 add = or_disjoint(f, rays[768 + sq]);
+  P = join32((u32)add * h + (u32)P, (u32)(add >> 32) * h + (u32)(P >> 32));
+  O = join32((u32)f * (0u - h) + (u32)O, (u32)(f >> 32) * (0u - h) + (u32)(O >> 32));
+  return has;
+}
+
+__device__ __forceinline__ void pair_book(PairSide& X, bool has) {
+  if (has) {
+    ++X.n;
+    X.passed = false;
+    X.fresh = false;
+    X.buf.x = X.buf.y;
+    X.buf.y = X.buf.z;
+    X.buf.z = X.buf.w;
+    if (X.n == X.empties) X.done = true;
+  } else if (!X.done) {
+    if (X.passed) X.done = true;
+    else X.passed = true;
+  }
+}
+
+// Returns the two results (+1 / 0 / -1 for each start position's side to
+// move; an inactive side returns 0) and adds both ply counts to *plies.
+__device__ __forceinline__ void playout_pair(u64 meX, u64 opX, u32 c0X, u32 c2X, bool actX,
+                                             u64 meY, u64 opY, u32 c0Y, u32 c2Y, bool actY,
+                                             uint2 key, u32 c1, const u64* __restrict__ rays,
+                                             u32* plies, int& rX, int& rY) {
+  PairSide X, Y;
+  pair_init(X, meX, opX, c0X, c2X, actX);
+  pair_init(Y, meY, opY, c0Y, c2Y, actY);
+  while (!(X.done && Y.done)) {
+    pair_refill(X, key, c1);
+    pair_refill(Y, key, c1);
+    const bool hx1 = pair_ply(meX, opX, X, rays);
+    const bool hy1 = pair_ply(meY, opY, Y, rays);
+    pair_book(X, hx1);
+    pair_book(Y, hy1);
+    if (X.done && Y.done) break;
+    pair_refill(X, key, c1);
+    pair_refill(Y, key, c1);
+    const bool hx2 = pair_ply(opX, meX, X, rays);
+    const bool hy2 = pair_ply(opY, meY, Y, rays);
+    pair_book(X, hx2);
+    pair_book(Y, hy2);
+  }
+  *plies += X.n + Y.n;
+  const int a = __popcll(meX), b = __popcll(opX), c = __popcll(meY), d = __popcll(opY);
+  rX = actX ? (a > b) - (a < b) : 0;
+  rY = actY ? (c > d) - (c < d) : 0;
+}
+
 }  // namespace mcts_dev
