@@ -249,7 +249,8 @@ typedef struct {
  *     iterations per tree per step: deterministic, bit-exact to the oracle;
  *     cpu_iters = 0 is the MCTS_BLOCK search bit for bit;
  *   time mode: steps until time_ms; cpu_iters > 0 lets the host iterate while
- *     each kernel runs (as many as fit), 0 = no CPU iterations.
+ *     each kernel runs (as many as fit; the caller's thread only drives the
+ *     GPU, the other cpu_threads - 1 iterate), 0 = no CPU iterations.
  * MCTS_BLOCK handle; n_trees in [1, 2^20]; threads_per_tree a multiple of 32
  * in [32, 1024]; cpu_threads in [1, 1024] host threads (the caller's thread
  * included); iteration mode: iterations * (threads_per_tree + cpu_iters)

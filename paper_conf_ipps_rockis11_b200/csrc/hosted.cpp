@@ -176,16 +176,23 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
           for (u32 j = 0; j < a.cpu_iters; ++j) cpu_iteration(trees[t], a, t);
         return;
       }
-      // time mode: round-robin over this thread's trees while the kernel runs
-      for (u32 t = w;; t += nthreads) {
-        if (t >= a.n_trees) t = w;
-        if (w == 0) {  // the driving thread polls the GPU
+      // time mode: the driving thread only polls the GPU, so the step ends as
+      // soon as the kernel does (a host iteration in progress on thread 0
+      // would hold the next step back); threads 1..T-1 iterate round-robin
+      // over the trees t = w - 1 (mod T - 1) while the kernel runs
+      if (w == 0) {
+        for (;;) {
           const int dn = gpu.done(gpu.ctx);
           if (dn != 0) {
             if (dn < 0) gpu_err = dn;
             P.gpu_done.store(1, std::memory_order_release);
+            return;
           }
         }
+      }
+      const u32 nw = nthreads - 1;
+      for (u32 t = w - 1;; t += nw) {
+        if (t >= a.n_trees) t = w - 1;
         if (P.gpu_done.load(std::memory_order_acquire)) break;
         cpu_iteration(trees[t], a, t);
       }

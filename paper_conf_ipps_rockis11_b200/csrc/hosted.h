@@ -13,7 +13,9 @@
 //      iterations with one host playout each on the SAME trees (streams c0 =
 //      tree id, c1 = 0x80000000 + the tree's CPU iteration count, c2 = 0):
 //      exactly cpu_iters per tree per step in iteration mode, as many as fit
-//      while the kernel runs in time mode (cpu_iters > 0);
+//      while the kernel runs in time mode (cpu_iters > 0; there thread 0 only
+//      drives the GPU and threads 1..T-1 iterate, so the host work never
+//      delays the next step);
 //   4. the host backpropagates the kernel's W/D/L along each tree's path.
 // Iteration mode is deterministic and bit-exact to the oracle's
 // orc_hybrid_search; with cpu_iters = 0 it is the block search bit for bit.
