@@ -137,12 +137,17 @@ block_search_kernel(TreePool T, SearchArgs a) {
 // ---------------------------------------------------------------------------
 // Leaf-parallel UCT: one tree; every thread of the grid
 // plays out from the same leaf each iteration. CTA 0's warp 0 owns the tree
-// (select/expand/backprop); the leaf is published through a small global
-// struct between two cooperative-groups grid barriers per iteration
-// (select -> sync -> simulate + per-CTA ballot reduce + atomics -> sync).
-// All CTAs are co-resident (cooperative launch). (Round 2 measured a
-// one-barrier hand-off — CTAs post their sums with one packed atomic and the
-// leader polls them — 20-27% slower from the opening.)
+// (select/expand/backprop). Per iteration: the leader publishes the leaf in a
+// small global struct and releases it with an iteration-stamped flag (thread
+// 0 of every other CTA spins on it with acquire loads, then a CTA barrier) ->
+// every thread simulates, CTAs ballot-reduce and add their wins/draws with
+// atomics -> one cooperative-groups grid barrier -> the leader backpropagates
+// and selects. All CTAs are co-resident (cooperative launch). Round 1 used a
+// grid barrier for the leaf hand-off too; after cg's grid.sync the CTAs' warp
+// 0 ran its playouts split in two (24.6 instead of 30.4 threads per
+// instruction, ncu r2z3), which doubled the batch latency: 53 -> 31 us per
+// iteration with the flag. MCTS_LEAF_POST (CTAs post packed
+// sums, the leader polls: no grid barrier at all) measured 4% slower.
 // ---------------------------------------------------------------------------
 // Tooling only (tools/leaf_compare.py variants): 1 = the leaf kernel skips the
 // playouts (every result a draw), so its iteration time is the serial part
@@ -151,11 +156,34 @@ block_search_kernel(TreePool T, SearchArgs a) {
 #define MCTS_LEAF_PROBE 0
 #endif
 
+#ifndef MCTS_LEAF_FLAG
+#define MCTS_LEAF_FLAG 1  // the leader publishes the leaf with a release flag instead of a grid barrier
+#endif
+#ifndef MCTS_LEAF_POST
+#define MCTS_LEAF_POST 0  // CTAs post (count, wins, draws) in one packed atomic; the leader polls it
+#endif
+
+
 struct LeafSync {
   u64 own, opp;
   u32 term, stop;
-  u32 wd[2][2];     // per-iteration-parity wins, draws
+  u32 wd[2][2];     // per-iteration-parity wins, draws (grid-barrier variant)
+  u32 flag;         // MCTS_LEAF_FLAG: iteration + 1 of the published leaf
+  u32 pad;
+  unsigned long long post[2];  // MCTS_LEAF_POST, per iteration parity: CTAs << 48 | wins << 24 | draws
 };
+
+__device__ __forceinline__ unsigned long long leaf_ld_relaxed64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ u32 leaf_ld_acquire(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 
 __global__ void __launch_bounds__(128)
 leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
@@ -187,9 +215,26 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
     if (leader) {
       if (it > 0) {
         const u32 par = (it - 1) & 1u;
+#if MCTS_LEAF_POST
+        // every CTA's (count, wins, draws) arrives in one packed word; lane 0
+        // polls it with relaxed loads (no acquire: that would drop the tree's
+        // lines from this SM's L1 on every poll) and clears the slot for
+        // iteration it + 1 before the next leaf is published
+        u32 W = 0, D = 0;
+        if (lane == 0) {
+          unsigned long long v;
+          while (((v = leaf_ld_relaxed64(&S->post[par])) >> 48) != gridDim.x) {}
+          W = (u32)(v >> 24) & 0xFFFFFFu;
+          D = (u32)v & 0xFFFFFFu;
+          S->post[par] = 0ULL;
+        }
+        W = __shfl_sync(kFull, W, 0);
+        D = __shfl_sync(kFull, D, 0);
+#else
         const u32 W = S->wd[par][0], D = S->wd[par][1];
         __syncwarp();
         if (lane == 0) { S->wd[par][0] = 0; S->wd[par][1] = 0; }
+#endif
         backprop(T, 0, &pc, s_depth, W, D, unit - W - D, lane);
       }
       u32 stop = 0;
@@ -207,11 +252,29 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
         }
       }
       if (lane == 0) S->stop = stop;
+#if MCTS_LEAF_FLAG
+      if (lane == 0) {
+        __threadfence();
+        asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(&S->flag), "r"(it + 1u) : "memory");
+      }
+#endif
     }
+#if MCTS_LEAF_FLAG
+    // one-to-all hand-off: the other CTAs wait for the leader's flag (their
+    // acquire also drops stale lines of S from their SM's L1); CTA 0 reads
+    // the leaf its own warp 0 wrote after the CTA barrier. The results still
+    // come back through the grid barrier below.
+    if (blockIdx.x != 0 && tid == 0) {
+      while (leaf_ld_acquire(&S->flag) != it + 1u) {}
+    }
+    __syncthreads();
+    __syncwarp();  // every warp enters the playouts converged (see the note above the kernel)
+#else
     grid.sync();
-    const u32 stop = S->stop;
-    const u64 own = S->own, opp = S->opp;
-    const u32 term = S->term;
+#endif
+    const u32 stop = __ldcg(&S->stop);
+    const u64 own = __ldcg(&S->own), opp = __ldcg(&S->opp);
+    const u32 term = __ldcg(&S->term);
     if (stop) break;
     int r;
     if (term) {
@@ -230,10 +293,17 @@ leaf_search_kernel(TreePool T, SearchArgs a, LeafSync* S) {
     __syncthreads();
     if (tid == 0) {
       const u32 par = it & 1u;
+#if MCTS_LEAF_POST
+      const unsigned long long w = s_w[0] + s_w[1] + s_w[2] + s_w[3], d = s_d[0] + s_d[1] + s_d[2] + s_d[3];
+      atomicAdd(&S->post[par], (1ULL << 48) | (w << 24) | d);
+#else
       atomicAdd(&S->wd[par][0], s_w[0] + s_w[1] + s_w[2] + s_w[3]);
       atomicAdd(&S->wd[par][1], s_d[0] + s_d[1] + s_d[2] + s_d[3]);
+#endif
     }
+#if !MCTS_LEAF_POST
     grid.sync();
+#endif
   }
   const u32 bp = __reduce_add_sync(kFull, plies);
   if (lane == 0 && bp) atomicAdd(reinterpret_cast<unsigned long long*>(a.stats) + 197, (unsigned long long)bp);

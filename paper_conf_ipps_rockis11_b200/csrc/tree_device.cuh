@@ -101,6 +101,35 @@ __device__ __forceinline__ double ucb_value(u32 w, u32 k, u32 unit, double ln_pa
   return __dadd_rn(exploit, explore);
 }
 
+#ifndef MCTS_REDUX_ARGMAX
+#define MCTS_REDUX_ARGMAX 1
+#endif
+
+// Warp argmax of (u, i): the largest u, the lowest i among equal u; lanes with
+// no candidate hold i = kNoChild (u = -inf). Returns the winning i in every
+// lane. With MCTS_REDUX_ARGMAX the doubles are mapped to order-preserving
+// 64-bit keys and reduced with three warp reductions (max of the high words,
+// max of the low words among the lanes that hold it, min index among the
+// lanes that hold both) instead of five rounds of shuffles; same result.
+__device__ __forceinline__ u32 warp_argmax(double u, u32 i) {
+#if MCTS_REDUX_ARGMAX
+  const unsigned long long b = (unsigned long long)__double_as_longlong(u);
+  const unsigned long long key = i == kNoChild ? 0ULL : ((b >> 63) ? ~b : (b | 0x8000000000000000ULL));
+  const u32 hi = (u32)(key >> 32), lo = (u32)key;
+  const u32 mhi = __reduce_max_sync(kFull, hi);
+  const u32 mlo = __reduce_max_sync(kFull, hi == mhi ? lo : 0u);
+  return __reduce_min_sync(kFull, (hi == mhi && lo == mlo) ? i : kNoChild);
+#else
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    const double ou = __shfl_xor_sync(kFull, u, off);
+    const u32 oi = __shfl_xor_sync(kFull, i, off);
+    if (ou > u || (ou == u && oi < i)) { u = ou; i = oi; }
+  }
+  return i;
+#endif
+}
+
 struct LeafInfo {
   u64 own, opp;
   u32 term;
@@ -155,12 +184,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
         bm = mc; bf = fc; bk = kc; bw = wc; bd = dc; bo = oc; bp = pc_; bl = lc;
       }
     }
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) {
-      const double ou = __shfl_xor_sync(kFull, best_u, off);
-      const u32 oi = __shfl_xor_sync(kFull, best_i, off);
-      if (ou > best_u || (ou == best_u && oi < best_i)) { best_u = ou; best_i = oi; }
-    }
+    best_i = warp_argmax(best_u, best_i);
     // child best_i was scored by lane best_i mod 32, whose own best it is
     const int src = (int)(best_i & 31u);
     v = first + best_i;
