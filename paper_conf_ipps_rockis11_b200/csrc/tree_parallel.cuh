@@ -190,15 +190,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
         best_u = u; best_i = i; best_meta = mc; best_first = fc; best_k = kk;
       }
     }
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) {
-      const double ou = __shfl_xor_sync(kFull, best_u, off);
-      const u32 oi = __shfl_xor_sync(kFull, best_i, off);
-      if (oi != kNoChild && (best_i == kNoChild || ou > best_u || (ou == best_u && oi < best_i))) {
-        best_u = ou;
-        best_i = oi;
-      }
-    }
+    best_i = warp_argmax(best_u, best_i);  // lanes without a published child hold kNoChild
     if (best_i == kNoChild) break;  // no child published yet: simulate from v
     const int src = (int)(best_i & 31u);
     v = first + best_i;
