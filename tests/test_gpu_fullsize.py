@@ -106,7 +106,7 @@ def test_search_4736_trees_of_32_reaches_selection(block, orc):
 @pytest.mark.parametrize("threads,iters,seed", [(16384, 40, 4), (65536, 20, 9)])
 def test_search_leaf_full_batch_reaches_selection(leaf, orc, threads, iters, seed):
     """configs[3] (1 tree x 16384 threads per leaf batch, 128 co-resident CTAs
-    with grid barriers) and the largest batch (65536) long enough that the
+    with a flag hand-off and a grid barrier) and the largest batch (65536) long enough that the
     multi-CTA select -> simulate -> backprop loop runs UCB selections."""
     root, c = _root_with_few_moves(orc, 15, 30, 40, 10)
     res = leaf.search(root, iterations=iters, n_trees=1, threads_per_tree=threads, seed=seed)
