@@ -265,6 +265,21 @@ def test_search_time_mode_invariants(mcts, orc):
     assert (legal >> res["best_move"]) & 1
 
 
+def test_search_leaf_time_mode_invariants(mcts_leaf, orc):
+    """configs[3] in time mode (flag hand-off + one grid barrier per iteration,
+    DESIGN.md §5): ~30 us per iteration, so 100 ms run thousands of iterations;
+    every iteration adds exactly one batch to the root."""
+    root = orc.gen_positions(21, 1, 10, 20)
+    res = mcts_leaf.search(root, time_ms=100.0, n_trees=1, threads_per_tree=16384, seed=6)
+    s = res["stats"]
+    assert res["iterations"] > 1000
+    assert s[195] == res["iterations"] * 16384
+    assert s[:65].sum() == s[195]
+    assert (s[65:130] + s[130:195] <= s[:65]).all()
+    own, opp = pkg.own_opp(root)
+    assert (orc.legal(own, opp) >> res["best_move"]) & 1
+
+
 def test_search_time_mode_pool_full(orc):
     """A tiny node pool fills up; the search keeps simulating without expanding."""
     m = pkg.Mcts(c_uct=1.0, scheme="block", max_nodes_per_tree=64, device=0)
