@@ -719,6 +719,26 @@ def main():
     e2e_s = max_over_ranks(time.perf_counter() - t0)
     barrier()
     e2e_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_s
+    # ---- the same steps pipelined through mcts_playouts_host_async (step i+1's
+    # copies and launch are enqueued while step i runs; every step still copies
+    # its leaves in and its counts and ply count out through pinned host memory)
+    h_outs = [torch.empty((N_LEAVES, 3), dtype=torch.int32).pin_memory() for _ in range(2)]
+    h_plies = torch.zeros(2, dtype=torch.int64).pin_memory()
+    for i in range(8):  # one call per staging slot (MCTS_HOST_ASYNC_SLOTS): allocation outside the timing
+        m.playouts_host_async(h_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, h_outs[i % 2].data_ptr(),
+                              h_plies.data_ptr() + 8 * (i % 2), stream)
+    stream.synchronize()
+    barrier()
+    t0 = time.perf_counter()
+    for i in range(e2e_steps):
+        m.playouts_host_async(h_leaves.data_ptr(), N_LEAVES, N_PER_LEAF, PLAYOUT_SEED, h_outs[i % 2].data_ptr(),
+                              h_plies.data_ptr() + 8 * (i % 2), stream)
+    stream.synchronize()
+    e2e_pipe_s = max_over_ranks(time.perf_counter() - t0)
+    barrier()
+    e2e_pipe_value = world * e2e_steps * N_LEAVES * N_PER_LEAF / e2e_pipe_s
+    if not torch.equal(h_outs[0], h_out):
+        raise RuntimeError("mcts_playouts_host_async and mcts_playouts disagree")
 
     log('# ---- opening-phase batch')
     # ---- the same kernel on an opening-phase batch (L in [0, 8] random plies:
@@ -869,7 +889,10 @@ def main():
         "roofline": roof,
         "e2e": {"value": e2e_value, "unit": "playouts/s",
                 "h2d_bytes_per_step": N_LEAVES * 24, "d2h_bytes_per_step": N_LEAVES * 12 + 8,
-                "api": "mcts_playouts (host buffers, pinned)"},
+                "api": "mcts_playouts (host buffers, pinned; synchronous per step)",
+                "pipelined": {"value": e2e_pipe_value, "unit": "playouts/s",
+                              "api": "mcts_playouts_host_async (host buffers, pinned; steps enqueued back "
+                                     "to back on one stream, one synchronisation at the end)"}},
         "gpu_launches": launches,
         "clocks": clocks,
         "opening_batch": opening_batch, "search": search, "leaf_search": leaf_search,

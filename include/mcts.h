@@ -157,6 +157,22 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
                           uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts,
                           uint64_t* out_plies);
 
+/* mcts_playouts with host buffers, asynchronous (a serving pipeline: step
+ * i + 1's copies and launch are enqueued while step i runs). Enqueues on
+ * `stream` the H2D copy of leaf_batch, the playouts, the D2H copy of the counts
+ * into out_counts and of the ply count into *out_plies, and returns without
+ * waiting; the results are valid once the stream has reached this point
+ * (cudaStreamSynchronize / an event). leaf_batch, out_counts and out_plies
+ * must be pinned host memory (cudaHostAlloc / torch pin_memory) and stay
+ * untouched until then; out_plies may be NULL. Same results as mcts_playouts.
+ * Device staging: a ring of MCTS_HOST_ASYNC_SLOTS slots per handle, reused in
+ * stream order, so every call on a handle must use the same stream. Leaves are
+ * not validated (as mcts_playouts_async). Errors: INVALID_ARGUMENT, OOM, CUDA. */
+#define MCTS_HOST_ASYNC_SLOTS 8
+mcts_status mcts_playouts_host_async(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
+                                     uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts,
+                                     uint64_t* out_plies, void* stream);
+
 /* Device-pointer / stream variant. d_leaves (device, n_leaves), d_out (device,
  * n_leaves, overwritten), d_plies (device uint64, nullable, ACCUMULATED into).
  * Streams use c0 = leaf_id_base + i so a batch split across GPUs by leaf range

@@ -23,7 +23,7 @@ MCTS_FLAG_CHECK_TREE = 1
 # every symbol include/mcts.h declares
 EXPORTS = (
     "mcts_create", "mcts_destroy", "mcts_playouts", "mcts_playouts_async", "mcts_search",
-    "mcts_search_async", "mcts_search_hybrid", "mcts_search_hosted", "mcts_playouts_ex_async", "mcts_best_move", "mcts_perft", "mcts_gen_positions_async", "mcts_ln_table",
+    "mcts_search_async", "mcts_search_hybrid", "mcts_search_hosted", "mcts_playouts_ex_async", "mcts_playouts_host_async", "mcts_best_move", "mcts_perft", "mcts_gen_positions_async", "mcts_ln_table",
     "mcts_status_string", "mcts_last_error", "mcts_version",
 )
 
@@ -90,6 +90,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
     L.mcts_playouts_async.restype = i32
     L.mcts_playouts_ex_async.argtypes = [vp, vp, u32, u32, u64, u32, u32, vp, vp, vp]
     L.mcts_playouts_ex_async.restype = i32
+    L.mcts_playouts_host_async.argtypes = [vp, vp, u32, u32, u64, vp, vp, vp]
+    L.mcts_playouts_host_async.restype = i32
     L.mcts_search_hosted.argtypes = [vp, P(Position), Budget, u32, u32, u64, u32, u32, P(RootStats), P(HostedInfo)]
     L.mcts_search_hosted.restype = i32
     L.mcts_search.argtypes = [vp, P(Position), Budget, u32, u32, u64, P(RootStats)]
@@ -183,6 +185,13 @@ class Mcts:
         self._check(self.L.mcts_playouts(self.h, leaves_ptr, n, n_per_leaf, seed, out_ptr,
                                          ctypes.byref(plies)))
         return int(plies.value)
+
+    def playouts_host_async(self, leaves_ptr: int, n: int, n_per_leaf: int, seed: int, out_ptr: int,
+                            plies_ptr: int = 0, stream=None):
+        """mcts_playouts_host_async on raw pinned host pointers: enqueued on
+        `stream`, valid after the stream is synchronised."""
+        self._check(self.L.mcts_playouts_host_async(self.h, leaves_ptr, n, n_per_leaf, seed, out_ptr,
+                                                    plies_ptr or None, _stream_ptr(stream)))
 
     # --- mcts_playouts_async (device pointers) ---------------------------
     def playouts_async(self, d_leaves_ptr: int, n_leaves: int, n_per_leaf: int, seed: int,

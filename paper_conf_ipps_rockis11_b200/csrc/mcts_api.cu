@@ -46,6 +46,11 @@ struct mcts_handle {
   size_t wdl_cap = 0;
   unsigned long long* d_plies = nullptr;
   unsigned long long* h_pin_plies = nullptr;
+  // mcts_playouts_host_async: ring of device staging slots, each one region
+  // [u32 work, u32 pad, u64 plies, n x WdlOut] followed by the leaves
+  void* d_async[MCTS_HOST_ASYNC_SLOTS] = {};
+  size_t async_cap[MCTS_HOST_ASYNC_SLOTS] = {};
+  uint32_t async_next = 0;
 
   // trees
   void* pool_mem = nullptr;
@@ -609,6 +614,7 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
+  for (int i = 0; i < MCTS_HOST_ASYNC_SLOTS; ++i) cudaFree(h->d_async[i]);
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
   if (h->h_pin_plies) cudaFreeHost(h->h_pin_plies);
@@ -706,6 +712,47 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
   CK(h, cudaMemcpyAsync(h->h_pin_plies, d_plies, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   CK(h, cudaStreamSynchronize(s));
   if (out_plies) *out_plies = *h->h_pin_plies;
+  return MCTS_OK;
+}
+
+mcts_status mcts_playouts_host_async(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
+                                     uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts,
+                                     uint64_t* out_plies, void* stream) {
+  if (!h) return MCTS_E_INVALID_ARGUMENT;
+  if (n_leaves && (!leaf_batch || !out_counts)) return fail(h, MCTS_E_INVALID_ARGUMENT, "NULL leaf_batch / out_counts");
+  if ((uint64_t)n_leaves * n_per_leaf / 32 > 0xFFFFFFF0ull)
+    return fail(h, MCTS_E_INVALID_ARGUMENT, "batch too large (>= 2^37 playouts)");
+  mcts_status st = check_device(h);
+  if (st) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n_leaves == 0) {
+    if (out_plies) *out_plies = 0;
+    return MCTS_OK;
+  }
+  constexpr size_t kHead = 16;  // u32 work, u32 pad, u64 plies
+  const size_t out_bytes = (size_t)n_leaves * sizeof(WdlOut);
+  const size_t leaves_off = (kHead + out_bytes + 255) & ~(size_t)255;
+  const size_t region = leaves_off + (size_t)n_leaves * sizeof(DevPosition);
+  const uint32_t slot = h->async_next++ % MCTS_HOST_ASYNC_SLOTS;
+  if (h->async_cap[slot] < region && h->d_async[slot]) {
+    // the slot's previous call may still be in flight on the stream
+    CK(h, cudaStreamSynchronize(s));
+  }
+  st = ensure(h, &h->d_async[slot], &h->async_cap[slot], region);
+  if (st) return st;
+  char* base = (char*)h->d_async[slot];
+  u32* work = (u32*)base;
+  uint64_t* d_plies = (uint64_t*)(base + 8);
+  mcts_wdl* d_out = (mcts_wdl*)(base + kHead);
+  mcts_position* d_leaves = (mcts_position*)(base + leaves_off);
+  CK(h, cudaMemsetAsync(base, 0, kHead + out_bytes, s));
+  CK(h, cudaMemcpyAsync(d_leaves, leaf_batch, (size_t)n_leaves * sizeof(DevPosition), cudaMemcpyHostToDevice, s));
+  if (n_per_leaf) {
+    st = launch_playouts(h, d_leaves, n_leaves, n_per_leaf, seed, 0u, 0u, d_out, d_plies, work, s);
+    if (st) return st;
+  }
+  CK(h, cudaMemcpyAsync(out_counts, d_out, out_bytes, cudaMemcpyDeviceToHost, s));
+  if (out_plies) CK(h, cudaMemcpyAsync(out_plies, d_plies, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   return MCTS_OK;
 }
 

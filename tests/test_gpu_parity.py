@@ -474,3 +474,29 @@ def test_playouts_pinned_host_buffers(mcts, orc):
     plies = mcts.playouts_host_ptr(h_in.data_ptr(), n, 7, 9, h_out2.data_ptr())
     want, wplies = orc.playouts(leaves, 7, seed=9)
     assert (h_out2.numpy() == want).all() and plies == wplies
+
+
+def test_playouts_host_async_pipelined(mcts, orc):
+    """mcts_playouts_host_async: twelve calls in flight on one stream (more than
+    the handle's 8 staging slots, so slots are reused in stream order), with
+    different seeds, batch sizes and output buffers, one synchronisation at the
+    end; every call bit-exact to the oracle, ply counts included. Zero
+    playouts per leaf and zero leaves give zeros."""
+    stream = torch.cuda.Stream()
+    leaves = orc.gen_positions(83, 200, 20, 40)
+    h_in = torch.from_numpy(leaves.view(np.int64).reshape(-1, 3).copy()).pin_memory()
+    calls = [(200 if i % 3 else 150, 24 + i, 100 + i) for i in range(12)]  # (n, per, seed)
+    outs = [torch.full((n, 3), -1, dtype=torch.int32).pin_memory() for n, _, _ in calls]
+    plies = torch.full((len(calls),), -1, dtype=torch.int64).pin_memory()
+    for i, (n, per, seed) in enumerate(calls):
+        mcts.playouts_host_async(h_in.data_ptr(), n, per, seed, outs[i].data_ptr(), plies.data_ptr() + 8 * i,
+                                 stream)
+    stream.synchronize()
+    for i, (n, per, seed) in enumerate(calls):
+        want, wplies = orc.playouts(leaves[:n], per, seed=seed)
+        assert (outs[i].numpy() == want).all() and int(plies[i]) == wplies, i
+    z = torch.full((200, 3), -1, dtype=torch.int32).pin_memory()
+    mcts.playouts_host_async(h_in.data_ptr(), 200, 0, 1, z.data_ptr(), plies.data_ptr(), stream)
+    mcts.playouts_host_async(h_in.data_ptr(), 0, 5, 1, z.data_ptr(), plies.data_ptr() + 8, stream)
+    stream.synchronize()
+    assert (z == 0).all() and int(plies[0]) == 0 and int(plies[1]) == 0
