@@ -11,7 +11,12 @@ playout streams (leaf_id_base = rank * 4096): weak scaling, no collective on
 the data path. The block-parallel search (configs[2] shape, a1-a11 incl. the
 NCCL root-stats allreduce at N>1), the leaf-parallel comparison (configs[3])
 and the NEXT-4 shared tree (1184 workers x 128 threads on one tree) are reported
-in the "search" / "leaf_search" / "tree_search" objects of the same line.
+in the "search" / "leaf_search" / "tree_search" objects of the same line
+(device-timed from a spin kernel's end, so host-side enqueue time stays out),
+the paper's CPU-managed trees in "hosted_search". "e2e" is the same batch
+through mcts_playouts with pinned host buffers, one synchronous call per step;
+"e2e.pipelined" the same steps through mcts_playouts_host_async, enqueued
+back to back with one synchronisation.
 
 Prints ONE JSON line on rank 0. See DESIGN.md §8 for every field.
 """
