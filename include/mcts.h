@@ -157,7 +157,7 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
                           uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts,
                           uint64_t* out_plies);
 
-/* mcts_playouts with host buffers, asynchronous (a serving pipeline: step
+/* mcts_playouts (PAPER.md L149-L153, L231-L237) with host buffers, asynchronous (a serving pipeline: step
  * i + 1's copies and launch are enqueued while step i runs). Enqueues on
  * `stream` the H2D copy of leaf_batch, the playouts, the D2H copy of the counts
  * into out_counts and of the ply count into *out_plies, and returns without
