@@ -165,9 +165,10 @@ mcts_status mcts_playouts(mcts_handle* h, const mcts_position* leaf_batch, uint3
  * (cudaStreamSynchronize / an event). leaf_batch, out_counts and out_plies
  * must be pinned host memory (cudaHostAlloc / torch pin_memory) and stay
  * untouched until then; out_plies may be NULL. Same results as mcts_playouts.
- * Device staging: a ring of MCTS_HOST_ASYNC_SLOTS slots per handle, reused in
- * stream order, so every call on a handle must use the same stream. Leaves are
- * not validated (as mcts_playouts_async). Errors: INVALID_ARGUMENT, OOM, CUDA. */
+ * Device staging: a ring of MCTS_HOST_ASYNC_SLOTS slots per handle; a slot's
+ * reuse waits (cudaStreamWaitEvent) for its previous call's copies, so calls
+ * may use different streams. Leaves are not validated (as
+ * mcts_playouts_async). Errors: INVALID_ARGUMENT, OOM, CUDA. */
 #define MCTS_HOST_ASYNC_SLOTS 8
 mcts_status mcts_playouts_host_async(mcts_handle* h, const mcts_position* leaf_batch, uint32_t n_leaves,
                                      uint32_t n_per_leaf, uint64_t seed, mcts_wdl* out_counts,

@@ -50,6 +50,7 @@ struct mcts_handle {
   // [u32 work, u32 pad, u64 plies, n x WdlOut] followed by the leaves
   void* d_async[MCTS_HOST_ASYNC_SLOTS] = {};
   size_t async_cap[MCTS_HOST_ASYNC_SLOTS] = {};
+  cudaEvent_t async_done[MCTS_HOST_ASYNC_SLOTS] = {};  // the slot's last D2H, for reuse from any stream
   uint32_t async_next = 0;
 
   // trees
@@ -614,7 +615,10 @@ void mcts_destroy(mcts_handle* h) {
   cudaFree(h->d_treesync);
   cudaFree(h->d_rays);
   cudaFree(h->d_work);
-  for (int i = 0; i < MCTS_HOST_ASYNC_SLOTS; ++i) cudaFree(h->d_async[i]);
+  for (int i = 0; i < MCTS_HOST_ASYNC_SLOTS; ++i) {
+    cudaFree(h->d_async[i]);
+    if (h->async_done[i]) cudaEventDestroy(h->async_done[i]);
+  }
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
   if (h->h_pin_plies) cudaFreeHost(h->h_pin_plies);
@@ -734,10 +738,13 @@ mcts_status mcts_playouts_host_async(mcts_handle* h, const mcts_position* leaf_b
   const size_t leaves_off = (kHead + out_bytes + 255) & ~(size_t)255;
   const size_t region = leaves_off + (size_t)n_leaves * sizeof(DevPosition);
   const uint32_t slot = h->async_next++ % MCTS_HOST_ASYNC_SLOTS;
+  if (!h->async_done[slot]) CK(h, cudaEventCreateWithFlags(&h->async_done[slot], cudaEventDisableTiming));
   if (h->async_cap[slot] < region && h->d_async[slot]) {
-    // the slot's previous call may still be in flight on the stream
-    CK(h, cudaStreamSynchronize(s));
+    // the slot's previous call may still be in flight: wait before freeing it
+    CK(h, cudaEventSynchronize(h->async_done[slot]));
   }
+  // the slot's previous call (on any stream) must have copied its results out
+  CK(h, cudaStreamWaitEvent(s, h->async_done[slot], 0));
   st = ensure(h, &h->d_async[slot], &h->async_cap[slot], region);
   if (st) return st;
   char* base = (char*)h->d_async[slot];
@@ -753,6 +760,7 @@ mcts_status mcts_playouts_host_async(mcts_handle* h, const mcts_position* leaf_b
   }
   CK(h, cudaMemcpyAsync(out_counts, d_out, out_bytes, cudaMemcpyDeviceToHost, s));
   if (out_plies) CK(h, cudaMemcpyAsync(out_plies, d_plies, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  CK(h, cudaEventRecord(h->async_done[slot], s));
   return MCTS_OK;
 }
 

@@ -477,12 +477,14 @@ def test_playouts_pinned_host_buffers(mcts, orc):
 
 
 def test_playouts_host_async_pipelined(mcts, orc):
-    """mcts_playouts_host_async: twelve calls in flight on one stream (more than
-    the handle's 8 staging slots, so slots are reused in stream order), with
-    different seeds, batch sizes and output buffers, one synchronisation at the
-    end; every call bit-exact to the oracle, ply counts included. Zero
-    playouts per leaf and zero leaves give zeros."""
-    stream = torch.cuda.Stream()
+    """mcts_playouts_host_async: twelve calls in flight on two alternating
+    streams (more than the handle's 8 staging slots, so slots are reused
+    across streams behind their previous call's event), with different seeds,
+    batch sizes and output buffers, one synchronisation at the end; every call
+    bit-exact to the oracle, ply counts included. Zero playouts per leaf and
+    zero leaves give zeros."""
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    stream = streams[0]
     leaves = orc.gen_positions(83, 200, 20, 40)
     h_in = torch.from_numpy(leaves.view(np.int64).reshape(-1, 3).copy()).pin_memory()
     calls = [(200 if i % 3 else 150, 24 + i, 100 + i) for i in range(12)]  # (n, per, seed)
@@ -490,8 +492,9 @@ def test_playouts_host_async_pipelined(mcts, orc):
     plies = torch.full((len(calls),), -1, dtype=torch.int64).pin_memory()
     for i, (n, per, seed) in enumerate(calls):
         mcts.playouts_host_async(h_in.data_ptr(), n, per, seed, outs[i].data_ptr(), plies.data_ptr() + 8 * i,
-                                 stream)
-    stream.synchronize()
+                                 streams[i % 2])
+    for st in streams:
+        st.synchronize()
     for i, (n, per, seed) in enumerate(calls):
         want, wplies = orc.playouts(leaves[:n], per, seed=seed)
         assert (outs[i].numpy() == want).all() and int(plies[i]) == wplies, i
