@@ -1,11 +1,12 @@
 // hosted.cpp — CPU-managed block-parallel trees with GPU simulation and the
 // hybrid CPU-GPU processing of PAPER.md §III-A (see hosted.h).
 //
-// Host threads own disjoint sets of trees (tree t belongs to thread t mod T;
-// thread 0 is the caller, which also drives the GPU). Each step is three
-// phases separated by spin barriers: select (every tree's GPU leaf into the
-// pinned leaf buffer) -> GPU playouts || CPU iterations on the same trees ->
-// backpropagation of the GPU results. The UCB arithmetic is R1's five IEEE
+// Host threads own disjoint sets of trees (thread 0 is the caller, which also
+// drives the GPU). The trees run in two halves pipelined on the GPU; per half
+// and step: select (its GPU leaves into the pinned leaf buffer) -> GPU
+// playouts || CPU iterations on the same trees -> backpropagation, phases
+// separated by spin barriers, and one half's host phases overlap the other
+// half's kernel (see run()). The UCB arithmetic is R1's five IEEE
 // round-to-nearest operations (the library is built with -ffp-contract=off).
 #include "hosted.h"
 #include "host_rules.h"
@@ -143,6 +144,8 @@ struct Pool {
   std::atomic<int> cmd{0};
   std::atomic<int> arrived{0};
   std::atomic<int> gpu_done{0};
+  std::atomic<int> slot{0};       // the half whose kernel the CPU phase overlaps
+  std::atomic<u32> lo{0}, hi{0};  // the phase's tree range
   std::atomic<u64> max_root_n{0};
 };
 
@@ -159,10 +162,24 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
   Pool P;
   int gpu_err = 0;
 
-  // the work of phase `c` for thread `w` (trees t = w, w + T, ...)
+  // The trees are processed in two halves that alternate on the GPU (one
+  // stream, so the device runs them back to back): while half A's kernel
+  // runs, the host selects half B's leaves and submits them, then runs the
+  // CPU iterations of half A, waits for A and backpropagates it, selects and
+  // submits A's next step, and so on. Every tree still sees select -> its
+  // kernel || its CPU iterations -> backprop, in that order and with the same
+  // streams, so results are unchanged; the host's sequential part
+  // now overlaps the other half's kernel instead of idling the GPU.
+  const u32 nh = a.n_trees >= 2 ? 2u : 1u;
+  const u32 split = nh == 2 ? (a.n_trees + 1) / 2 : a.n_trees;
+  const u32 lo_of[2] = {0u, split}, hi_of[2] = {split, a.n_trees};
+
+  // the work of phase `c` on trees [P.lo, P.hi) for thread `w` (trees lo + w,
+  // lo + w + T, ...; CPU iterations in time mode: threads 1..T-1)
   auto work = [&](int c, u32 w) {
+    const u32 lo = P.lo.load(std::memory_order_relaxed), hi = P.hi.load(std::memory_order_relaxed);
     if (c == kSelect) {
-      for (u32 t = w; t < a.n_trees; t += nthreads) {
+      for (u32 t = lo + w; t < hi; t += nthreads) {
         Tree& T = trees[t];
         bool e = false;
         const u32 v = select_expand(T, a, T.gpath, &e);
@@ -172,17 +189,18 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
     } else if (c == kCpu) {
       if (a.cpu_iters == 0) return;
       if (!timed) {
-        for (u32 t = w; t < a.n_trees; t += nthreads)
+        for (u32 t = lo + w; t < hi; t += nthreads)
           for (u32 j = 0; j < a.cpu_iters; ++j) cpu_iteration(trees[t], a, t);
         return;
       }
-      // time mode: the driving thread only polls the GPU, so the step ends as
-      // soon as the kernel does (a host iteration in progress on thread 0
-      // would hold the next step back); threads 1..T-1 iterate round-robin
-      // over the trees t = w - 1 (mod T - 1) while the kernel runs
+      // time mode: the driving thread only polls the GPU, so the half ends as
+      // soon as its kernel does (a host iteration in progress on thread 0
+      // would hold the pipeline back); threads 1..T-1 iterate round-robin
+      // over the half's trees while the kernel runs
       if (w == 0) {
+        const int slot = P.slot.load(std::memory_order_relaxed);
         for (;;) {
-          const int dn = gpu.done(gpu.ctx);
+          const int dn = gpu.done(gpu.ctx, slot);
           if (dn != 0) {
             if (dn < 0) gpu_err = dn;
             P.gpu_done.store(1, std::memory_order_release);
@@ -191,14 +209,15 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
         }
       }
       const u32 nw = nthreads - 1;
-      for (u32 t = w - 1;; t += nw) {
-        if (t >= a.n_trees) t = w - 1;
+      if (lo + w - 1 >= hi) return;
+      for (u32 t = lo + w - 1;; t += nw) {
+        if (t >= hi) t = lo + w - 1;
         if (P.gpu_done.load(std::memory_order_acquire)) break;
         cpu_iteration(trees[t], a, t);
       }
     } else if (c == kBackprop) {
       u64 mx = 0;
-      for (u32 t = w; t < a.n_trees; t += nthreads) {
+      for (u32 t = lo + w; t < hi; t += nthreads) {
         Tree& T = trees[t];
         const WdlRec r = gpu.wdl[t];
         backprop(T, T.gpath, a.unit, r.wins, r.draws, r.losses);
@@ -226,37 +245,63 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
       }
     });
   }
-  auto phase = [&](int c) {  // run phase c on every thread (the caller is thread 0)
+  auto phase = [&](int c, u32 half) {  // run phase c on half `half` on every thread (the caller is thread 0)
+    P.lo.store(lo_of[half], std::memory_order_relaxed);
+    P.hi.store(hi_of[half], std::memory_order_relaxed);
     P.arrived.store(0, std::memory_order_relaxed);
     P.cmd.store(c, std::memory_order_relaxed);
     P.gen.fetch_add(1, std::memory_order_acq_rel);
     work(c, 0);
     while (P.arrived.load(std::memory_order_acquire) < (int)nthreads - 1) std::this_thread::yield();
   };
-
-  u64 s = 0;
-  for (; s < a.steps; ++s) {
-    if (timed && now_ns() >= a.deadline_ns) break;
-    // the ln table covers every parent count this step's selections can read
-    // (at most the root's count plus the CPU iterations of the step)
-    if (P.max_root_n.load() + (timed ? 1000000ull : (u64)a.cpu_iters) >= a.lnT_size) break;
+  // another step may start: budget, deadline, and the ln table covers every
+  // parent count its selections can read (the root's count plus the step's
+  // CPU iterations)
+  auto may_start = [&](u64 step) {
+    if (step >= a.steps) return false;
+    if (timed && now_ns() >= a.deadline_ns) return false;
+    return P.max_root_n.load() + (timed ? 1000000ull : (u64)a.cpu_iters) < a.lnT_size;
+  };
+  auto launch = [&](u32 half, u64 step) {  // select the half's leaves and submit its kernel
     const int64_t t0 = now_ns();
-    phase(kSelect);
-    const int64_t t1 = now_ns();
-    if (gpu.submit(gpu.ctx, a.n_trees, (u32)s) < 0) { gpu_err = -1; break; }
+    phase(kSelect, half);
+    info->select_ms += (now_ns() - t0) * 1e-6;
+    if (gpu.submit(gpu.ctx, lo_of[half], hi_of[half] - lo_of[half], (u32)step, (int)half) < 0) gpu_err = -1;
+    return gpu_err == 0;
+  };
+  auto finish = [&](u32 half) {  // CPU iterations while its kernel runs, then its backprop
+    const int64_t t0 = now_ns();
+    P.slot.store((int)half, std::memory_order_relaxed);
     P.gpu_done.store(0, std::memory_order_release);
-    phase(kCpu);
-    if (!P.gpu_done.load(std::memory_order_acquire)) {
-      const int r = gpu.wait(gpu.ctx);
+    phase(kCpu, half);
+    if (!gpu_err && !P.gpu_done.load(std::memory_order_acquire)) {
+      const int r = gpu.wait(gpu.ctx, (int)half);
       if (r < 0) gpu_err = r;
     }
-    if (gpu_err) break;
-    const int64_t t2 = now_ns();
-    phase(kBackprop);
-    const int64_t t3 = now_ns();
-    info->select_ms += (t1 - t0) * 1e-6;
-    info->gpu_ms += (t2 - t1) * 1e-6;
-    info->backprop_ms += (t3 - t2) * 1e-6;
+    if (gpu_err) return false;
+    const int64_t t1 = now_ns();
+    phase(kBackprop, half);
+    info->gpu_ms += (t1 - t0) * 1e-6;
+    info->backprop_ms += (now_ns() - t1) * 1e-6;
+    return true;
+  };
+
+  u64 s = 0;
+  if (may_start(0) && launch(0, 0)) {
+    for (;;) {  // step s: half 0 is in flight
+      if (nh == 2 && !launch(1, s)) break;
+      if (!finish(0)) break;
+      if (nh == 2) {
+        const bool more = may_start(s + 1);
+        if (more && !launch(0, s + 1)) break;
+        if (!finish(1)) break;
+        ++s;
+        if (!more) break;
+      } else {
+        ++s;
+        if (!may_start(s) || !launch(0, s)) break;
+      }
+    }
   }
   P.cmd.store(kExit, std::memory_order_relaxed);
   P.gen.fetch_add(1, std::memory_order_acq_rel);

@@ -32,15 +32,17 @@ struct WdlRec {  // layout of mcts_wdl
   uint32_t wins, draws, losses;
 };
 
-// The GPU side, provided by mcts_api.cu: submit() copies n leaves (pinned
-// host) to the device, launches the playouts kernel for step `step` and copies
-// the W/D/L back into the pinned `wdl` buffer, all asynchronously; done()
-// polls (1 = finished, 0 = running, < 0 = CUDA error); wait() blocks.
+// The GPU side, provided by mcts_api.cu: submit() copies the leaves of trees
+// [first, first + n) (pinned host) to the device, launches the playouts kernel
+// for them at step `step` (streams c0 = tree id) and copies their W/D/L back
+// into the pinned `wdl` buffer, all asynchronously, completion tracked in
+// `slot` (0 or 1: the two pipelined halves, run in submission order); done()
+// polls a slot (1 = finished, 0 = running, < 0 = CUDA error); wait() blocks.
 struct Gpu {
   void* ctx;
-  int (*submit)(void* ctx, uint32_t n, uint32_t step);
-  int (*done)(void* ctx);
-  int (*wait)(void* ctx);
+  int (*submit)(void* ctx, uint32_t first, uint32_t n, uint32_t step, int slot);
+  int (*done)(void* ctx, int slot);
+  int (*wait)(void* ctx, int slot);
   LeafRec* leaves;    // pinned, n_trees
   const WdlRec* wdl;  // pinned, n_trees
 };

@@ -80,7 +80,8 @@ struct mcts_handle {
   mcts_position* h_pin_leaves = nullptr;
   mcts_wdl* h_pin_wdl = nullptr;
   size_t pin_cap = 0;
-  cudaEvent_t step_event = nullptr;
+  cudaEvent_t step_event[2] = {};  // the two pipelined halves
+  cudaStream_t stream2 = nullptr;  // the second half's stream (its kernels overlap the first half's)
 };
 
 namespace {
@@ -488,34 +489,37 @@ struct HostedGpu {
   cudaError_t err;
 };
 
-int hosted_submit(void* ctx, uint32_t n, uint32_t step) {
+int hosted_submit(void* ctx, uint32_t first, uint32_t n, uint32_t step, int slot) {
   HostedGpu* g = (HostedGpu*)ctx;
   mcts_handle* h = g->h;
-  cudaStream_t s = h->stream;
-  cudaError_t e = cudaMemcpyAsync(g->d_leaves, h->h_pin_leaves, (size_t)n * sizeof(mcts_position),
+  // one stream per half: a half's kernel can start while the other half's is
+  // still running (each fills part of the SMs; together the whole GPU)
+  cudaStream_t s = slot == 0 ? h->stream : h->stream2;
+  cudaError_t e = cudaMemcpyAsync(g->d_leaves + first, h->h_pin_leaves + first, (size_t)n * sizeof(mcts_position),
                                   cudaMemcpyHostToDevice, s);
-  if (e == cudaSuccess &&
-      mcts_playouts_ex_async(h, g->d_leaves, n, g->unit, g->seed, 0u, step, g->d_wdl, (uint64_t*)g->d_plies, s))
+  if (e == cudaSuccess && mcts_playouts_ex_async(h, g->d_leaves + first, n, g->unit, g->seed, first, step,
+                                                 g->d_wdl + first, (uint64_t*)g->d_plies, s))
     e = cudaErrorLaunchFailure;
   if (e == cudaSuccess)
-    e = cudaMemcpyAsync(h->h_pin_wdl, g->d_wdl, (size_t)n * sizeof(mcts_wdl), cudaMemcpyDeviceToHost, s);
-  if (e == cudaSuccess) e = cudaEventRecord(h->step_event, s);
+    e = cudaMemcpyAsync(h->h_pin_wdl + first, g->d_wdl + first, (size_t)n * sizeof(mcts_wdl),
+                        cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaEventRecord(h->step_event[slot], s);
   g->err = e;
   return e == cudaSuccess ? 0 : -1;
 }
 
-int hosted_done(void* ctx) {
+int hosted_done(void* ctx, int slot) {
   HostedGpu* g = (HostedGpu*)ctx;
-  const cudaError_t e = cudaEventQuery(g->h->step_event);
+  const cudaError_t e = cudaEventQuery(g->h->step_event[slot]);
   if (e == cudaSuccess) return 1;
   if (e == cudaErrorNotReady) return 0;
   g->err = e;
   return -1;
 }
 
-int hosted_wait(void* ctx) {
+int hosted_wait(void* ctx, int slot) {
   HostedGpu* g = (HostedGpu*)ctx;
-  const cudaError_t e = cudaEventSynchronize(g->h->step_event);
+  const cudaError_t e = cudaEventSynchronize(g->h->step_event[slot]);
   if (e != cudaSuccess) { g->err = e; return -1; }
   return 0;
 }
@@ -622,7 +626,12 @@ void mcts_destroy(mcts_handle* h) {
   if (h->h_pin_leaves) cudaFreeHost(h->h_pin_leaves);
   if (h->h_pin_wdl) cudaFreeHost(h->h_pin_wdl);
   if (h->h_pin_plies) cudaFreeHost(h->h_pin_plies);
-  if (h->step_event) cudaEventDestroy(h->step_event);
+  for (cudaEvent_t& ev : h->step_event)
+    if (ev) cudaEventDestroy(ev);
+  if (h->stream2) {
+    cudaStreamSynchronize(h->stream2);
+    cudaStreamDestroy(h->stream2);
+  }
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
@@ -887,7 +896,9 @@ mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_b
     CK(h, cudaHostAlloc((void**)&h->h_pin_wdl, (size_t)n_trees * sizeof(mcts_wdl), cudaHostAllocDefault));
     h->pin_cap = n_trees;
   }
-  if (!h->step_event) CK(h, cudaEventCreateWithFlags(&h->step_event, cudaEventDisableTiming));
+  for (cudaEvent_t& ev : h->step_event)
+    if (!ev) CK(h, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  if (!h->stream2) CK(h, cudaStreamCreateWithFlags(&h->stream2, cudaStreamNonBlocking));
   void* p = h->d_leaves;
   st = ensure(h, &p, &h->leaves_cap, (size_t)n_trees * sizeof(DevPosition));
   if (st) return st;
@@ -895,6 +906,9 @@ mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_b
   st = ensure(h, &h->d_wdl, &h->wdl_cap, (size_t)n_trees * sizeof(WdlOut));
   if (st) return st;
   CK(h, cudaMemsetAsync(h->d_plies, 0, sizeof(unsigned long long), h->stream));
+  // the second half's stream starts behind the zeroed ply counter
+  CK(h, cudaEventRecord(h->step_event[1], h->stream));
+  CK(h, cudaStreamWaitEvent(h->stream2, h->step_event[1], 0));
 
   HostedGpu g{h, seed, threads_per_tree, (mcts_position*)h->d_leaves, (mcts_wdl*)h->d_wdl, h->d_plies, cudaSuccess};
   mcts_hosted::Gpu gpu{&g, hosted_submit, hosted_done, hosted_wait,
@@ -918,6 +932,7 @@ mcts_status mcts_search_hosted(mcts_handle* h, const mcts_position* root, mcts_b
   long long hs[MCTS_STATS_LEN];
   mcts_hosted::Info hi;
   const int r = mcts_hosted::run(a, gpu, (int64_t*)hs, &hi);
+  cudaStreamSynchronize(h->stream2);
   if (r < 0) {
     cudaStreamSynchronize(h->stream);
     return cuda_fail(h, g.err == cudaSuccess ? cudaErrorUnknown : g.err, "mcts_search_hosted: GPU step");

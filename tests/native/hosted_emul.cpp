@@ -14,9 +14,9 @@ using namespace mcts_hosted;
 namespace {
 struct Ctx { LeafRec* leaves; WdlRec* wdl; uint64_t seed; uint32_t unit; uint64_t plies; };
 
-int submit(void* c, uint32_t n, uint32_t step) {
+int submit(void* c, uint32_t first, uint32_t n, uint32_t step, int) {
   Ctx* x = (Ctx*)c;
-  for (uint32_t t = 0; t < n; ++t) {
+  for (uint32_t t = first; t < first + n; ++t) {
     uint32_t w = 0, d = 0, l = 0;
     for (uint32_t j = 0; j < x->unit; ++j) {
       const int r = host_rules::playout(x->leaves[t].black, x->leaves[t].white, x->seed, t, step, j, &x->plies);
@@ -26,8 +26,8 @@ int submit(void* c, uint32_t n, uint32_t step) {
   }
   return 0;
 }
-int done(void*) { return 1; }
-int wait(void*) { return 0; }
+int done(void*, int) { return 1; }
+int wait(void*, int) { return 0; }
 }  // namespace
 
 extern "C" int hosted_emul(uint64_t own, uint64_t opp, uint32_t n_trees, uint32_t unit, uint64_t steps,
