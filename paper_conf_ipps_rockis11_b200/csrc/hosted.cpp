@@ -26,43 +26,23 @@ using namespace host_rules;
 
 int64_t now_ns() { return std::chrono::steady_clock::now().time_since_epoch().count(); }
 
-// Node storage, split by use so that selection touches one small record per
-// child: Hot (24 B) holds what a selection step reads (n, w of every child;
-// first, nchild, limit, term of the chosen one), Cold the board and the draws.
-// A child block is contiguous, so one level's UCB pass reads ~4 cache lines
-// and the chosen child's control fields come with it (round 1's one vector
-// per field cost two dependent cache misses per level).
-struct Hot {
-  u64 n, w;
-  u32 first;
-  uint8_t nchild, limit, move, term;
-};
-struct Cold {
-  u64 own, opp, lg, d;
-};
-
 struct Tree {
-  std::vector<Hot> hot;
-  std::vector<Cold> cold;
+  std::vector<u64> own, opp, lg, n, w, d;
+  std::vector<u32> first;
+  std::vector<uint8_t> nchild, limit, move, term;
   std::vector<u32> gpath, cpath;  // the pending GPU leaf's path; scratch for CPU iterations
   u64 cpu_count = 0, cpu_plies = 0, cpu_depth = 0, cpu_nodes = 0, gpu_nodes = 0;
   u64 depth_sum = 0, iterations = 0;
 
-  void set(u32 s, u64 o, u64 p, u32 mv) {
+  u32 add(u64 o, u64 p, u32 mv) {
     const u64 l = legal(o, p);
     const bool t = l == 0 && legal(p, o) == 0;
-    Hot& h = hot[s];
-    h.n = 0; h.w = 0; h.first = 0xFFFFFFFFu; h.nchild = 0;
-    h.limit = t ? 0 : (l ? (uint8_t)popc(l) : 1);
-    h.move = (uint8_t)mv; h.term = t ? 1 : 0;
-    cold[s] = Cold{o, p, l, 0};
-  }
-  u32 add(u64 o, u64 p, u32 mv) {
-    hot.push_back(Hot{});
-    cold.push_back(Cold{});
-    const u32 s = (u32)(hot.size() - 1);
-    set(s, o, p, mv);
-    return s;
+    own.push_back(o); opp.push_back(p); lg.push_back(l);
+    n.push_back(0); w.push_back(0); d.push_back(0);
+    first.push_back(0xFFFFFFFFu); nchild.push_back(0);
+    limit.push_back(t ? 0 : (l ? (uint8_t)popc(l) : 1));
+    move.push_back((uint8_t)mv); term.push_back(t ? 1 : 0);
+    return (u32)(own.size() - 1);
   }
 };
 
@@ -78,51 +58,47 @@ inline double ucb(u64 w, u64 n, double lnN, double C) {
 // Selection (L157-L178; a pending child, n = 0, is unvisited: taken first)
 // and expansion (L179-L182: the lowest-index untried move or the pass child)
 // of one iteration; the path root..leaf goes to `path`. Returns the leaf.
-// While a level's children are scored, each fully expanded child's own child
-// block is prefetched, so the next level's records are on their way before
-// the winner is known.
 u32 select_expand(Tree& T, const Args& a, std::vector<u32>& path, bool* expanded) {
   path.clear();
   u32 v = 0;
   path.push_back(v);
-  const Hot* H = T.hot.data();
-  while (!H[v].term && H[v].nchild >= H[v].limit) {
-    const u32 f = H[v].first;
-    const u32 nch = H[v].nchild;
-    const double lnN = a.lnT[H[v].n];
+  while (!T.term[v] && T.nchild[v] >= T.limit[v]) {
+    const u32 f = T.first[v];
+    const double lnN = a.lnT[T.n[v]];
     u32 best = f;
     double bu = -INFINITY;
-    for (u32 i = 0; i < nch; ++i) {
-      const Hot& c = H[f + i];
-      if (c.nchild && c.nchild >= c.limit) __builtin_prefetch(&H[c.first]);
-      if (c.n == 0) { best = f + i; break; }
-      const double u = ucb(c.w, c.n, lnN, a.C);
-      if (u > bu) { bu = u; best = f + i; }
+    for (u32 i = 0; i < T.nchild[v]; ++i) {
+      const u32 c = f + i;
+      if (T.n[c] == 0) { best = c; break; }
+      const double u = ucb(T.w[c], T.n[c], lnN, a.C);
+      if (u > bu) { bu = u; best = c; }
     }
     v = best;
     path.push_back(v);
   }
   *expanded = false;
-  if (!T.hot[v].term) {
-    if (T.hot[v].nchild == 0) {  // reserve the children's contiguous block
-      const u32 lim = T.hot[v].limit;
-      const u32 f = (u32)T.hot.size();
-      T.hot.resize(f + lim, Hot{});
-      T.cold.resize(f + lim, Cold{});
-      T.hot[v].first = f;
+  if (!T.term[v]) {
+    if (T.nchild[v] == 0) {  // reserve the children's contiguous block
+      const u32 lim = T.limit[v];
+      const u32 f = (u32)T.own.size();
+      for (u32 i = 0; i < lim; ++i) T.add(0, 0, 0);
+      T.first[v] = f;
     }
-    const u32 c = T.hot[v].first + T.hot[v].nchild;
-    const u64 o = T.cold[v].own, p = T.cold[v].opp, l = T.cold[v].lg;
+    const u32 c = T.first[v] + T.nchild[v];
+    const u64 o = T.own[v], p = T.opp[v], l = T.lg[v];
     u64 co, cp;
     u32 mv;
     if (l == 0) { co = p; cp = o; mv = 64; }
     else {
-      const int sq = kth_bit(l, T.hot[v].nchild);
+      const int sq = kth_bit(l, T.nchild[v]);
       const u64 fl = flips(sq, o, p);
       co = p & ~fl; cp = o | fl | (1ULL << sq); mv = (u32)sq;
     }
-    T.set(c, co, cp, mv);
-    T.hot[v].nchild += 1;
+    const u64 cl = legal(co, cp);
+    const bool ct = cl == 0 && legal(cp, co) == 0;
+    T.own[c] = co; T.opp[c] = cp; T.lg[c] = cl; T.move[c] = (uint8_t)mv; T.term[c] = ct ? 1 : 0;
+    T.limit[c] = ct ? 0 : (cl ? (uint8_t)popc(cl) : 1);
+    T.nchild[v] += 1;
     path.push_back(c);
     v = c;
     *expanded = true;
@@ -136,7 +112,7 @@ void backprop(Tree& T, const std::vector<u32>& path, u64 count, u64 W, u64 D, u6
   u64 mover = Lo, other = W;
   for (size_t i = path.size(); i-- > 0;) {
     const u32 x = path[i];
-    T.hot[x].n += count; T.hot[x].w += mover; T.cold[x].d += D;
+    T.n[x] += count; T.w[x] += mover; T.d[x] += D;
     std::swap(mover, other);
   }
 }
@@ -147,11 +123,11 @@ void cpu_iteration(Tree& T, const Args& a, u32 t) {
   const u32 v = select_expand(T, a, T.cpath, &e);
   T.cpu_nodes += e ? 1 : 0;
   int r;
-  if (T.hot[v].term) {
-    const int x = popc(T.cold[v].own), y = popc(T.cold[v].opp);
+  if (T.term[v]) {
+    const int x = popc(T.own[v]), y = popc(T.opp[v]);
     r = (x > y) - (x < y);
   } else {
-    r = playout(T.cold[v].own, T.cold[v].opp, a.seed, a.tree_id_base + t, 0x80000000u + (u32)T.cpu_count, 0u,
+    r = playout(T.own[v], T.opp[v], a.seed, a.tree_id_base + t, 0x80000000u + (u32)T.cpu_count, 0u,
                 &T.cpu_plies);
   }
   backprop(T, T.cpath, 1, r > 0, r == 0, r < 0);
@@ -180,7 +156,7 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
   *info = Info{};
   std::vector<Tree> trees(a.n_trees);
   for (Tree& T : trees) T.add(a.own, a.opp, 0xFF);
-  if (a.n_trees == 0 || trees[0].hot[0].term) return 0;
+  if (a.n_trees == 0 || trees[0].term[0]) return 0;
   const u32 nthreads = std::max<u32>(1, std::min<u32>(a.threads, a.n_trees));
   const bool timed = a.deadline_ns != 0;
   Pool P;
@@ -208,7 +184,7 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
         bool e = false;
         const u32 v = select_expand(T, a, T.gpath, &e);
         T.gpu_nodes += e ? 1 : 0;
-        gpu.leaves[t] = LeafRec{T.cold[v].own, T.cold[v].opp, 0u, 0u};  // black = side to move: to_move 0
+        gpu.leaves[t] = LeafRec{T.own[v], T.opp[v], 0u, 0u};  // black = side to move: to_move 0
       }
     } else if (c == kCpu) {
       if (a.cpu_iters == 0) return;
@@ -247,7 +223,7 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
         backprop(T, T.gpath, a.unit, r.wins, r.draws, r.losses);
         T.depth_sum += T.gpath.size() - 1;
         T.iterations += 1;
-        mx = std::max<u64>(mx, T.hot[0].n);
+        mx = std::max<u64>(mx, T.n[0]);
       }
       u64 cur = P.max_root_n.load();
       while (mx > cur && !P.max_root_n.compare_exchange_weak(cur, mx)) {}
@@ -334,14 +310,14 @@ int run(const Args& a, const Gpu& gpu, int64_t* stats, Info* info) {
 
   info->steps = s;
   for (const Tree& T : trees) {
-    const u32 f = T.hot[0].first;
-    for (u32 i = 0; i < T.hot[0].nchild; ++i) {
+    const u32 f = T.first[0];
+    for (u32 i = 0; i < T.nchild[0]; ++i) {
       const u32 c = f + i;
-      stats[T.hot[c].move] += (int64_t)T.hot[c].n;
-      stats[65 + T.hot[c].move] += (int64_t)T.hot[c].w;
-      stats[130 + T.hot[c].move] += (int64_t)T.cold[c].d;
+      stats[T.move[c]] += (int64_t)T.n[c];
+      stats[65 + T.move[c]] += (int64_t)T.w[c];
+      stats[130 + T.move[c]] += (int64_t)T.d[c];
     }
-    stats[195] += (int64_t)T.hot[0].n;
+    stats[195] += (int64_t)T.n[0];
     stats[196] += (int64_t)T.iterations;
     stats[197] += (int64_t)T.cpu_plies;  // + the kernel's plies (counted on the device)
     stats[198] += (int64_t)T.depth_sum;
