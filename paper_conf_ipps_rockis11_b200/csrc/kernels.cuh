@@ -48,6 +48,10 @@ struct SearchArgs {
 };
 
 
+#ifndef MCTS_BLOCK_BOARDS
+#define MCTS_BLOCK_BOARDS false  // block kernel: read the chosen leaf's board after the descent (fewer registers)
+#endif
+
 template <int MAX_THREADS, int MIN_BLOCKS>
 __global__ void __launch_bounds__(MAX_THREADS, MIN_BLOCKS)
 block_search_kernel(TreePool T, SearchArgs a) {
@@ -89,7 +93,7 @@ block_search_kernel(TreePool T, SearchArgs a) {
         }
         stop = __shfl_sync(kFull, stop, 0);
         if (!stop) {
-          const LeafInfo L = select_expand(T, base, &pc, &s_slot_used, a.lnT, unit, a.C, lane, s_rays);
+          const LeafInfo L = select_expand<MCTS_BLOCK_BOARDS>(T, base, &pc, &s_slot_used, a.lnT, unit, a.C, lane, s_rays);
           if (lane == 0) {
             s_own = L.own; s_opp = L.opp; s_term = L.term; s_depth = L.depth;
             depth_sum += (unsigned)L.depth;

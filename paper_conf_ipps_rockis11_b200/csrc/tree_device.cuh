@@ -151,6 +151,7 @@ struct LeafInfo {
 // the root comes from the cache, and the expansion needs no read at all —
 // instead of the five dependent reads per level, a root read and a board read
 // of round 1.
+template <bool BOARDS = true>  // false: the chosen node's board is read once after the descent
 __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base, PathCache* pc,
                                                   u32* slot_used, const double* __restrict__ lnT,
                                                   u32 unit, double C, int lane,
@@ -177,7 +178,8 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
     for (u32 i = (u32)lane; i < nch; i += 32u) {
       const size_t c = base + first + i;
       const u32 wc = T.w[c], kc = T.k[c], dc = T.d[c], mc = T.meta[c], fc = T.first[c];
-      const u64 oc = T.own[c], pc_ = T.opp[c], lc = T.legal[c];
+      u64 oc = 0, pc_ = 0, lc = 0;
+      if (BOARDS) { oc = T.own[c]; pc_ = T.opp[c]; lc = T.legal[c]; }
       const double u = ucb_value(wc, kc, unit, lnp, C);
       if (u > best_u) {
         best_u = u; best_i = i;
@@ -192,9 +194,11 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
     first = __shfl_sync(kFull, bf, src);
     kv = __shfl_sync(kFull, bk, src);
     const u32 wv = __shfl_sync(kFull, bw, src), dv = __shfl_sync(kFull, bd, src);
-    own = __shfl_sync(kFull, bo, src);
-    opp = __shfl_sync(kFull, bp, src);
-    lg = __shfl_sync(kFull, bl, src);
+    if (BOARDS) {
+      own = __shfl_sync(kFull, bo, src);
+      opp = __shfl_sync(kFull, bp, src);
+      lg = __shfl_sync(kFull, bl, src);
+    }
     ++depth;
     if (lane == 0) { pc->node[depth] = v; pc->k[depth] = kv; pc->w[depth] = wv; pc->d[depth] = dv; }
   }
@@ -204,6 +208,11 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
   L.refused = 0;
   u32 c = kNoChild;
   u32 term = meta_term(meta) ? 1u : 0u;
+  if (!BOARDS && depth > 0 && lane == 0) {
+    own = T.own[base + v];
+    opp = T.opp[base + v];
+    lg = T.legal[base + v];
+  }
   if (lane == 0 && !term) {
     const u32 nch = meta_nchild(meta), limit = meta_limit(meta);
     u32 f0 = first;
