@@ -60,3 +60,14 @@ def test_no_cpu_fallback_without_gpu():
     with pytest.raises(pkg.MctsError) as ei:
         pkg.Mcts()
     assert ei.value.status == -5  # MCTS_E_NO_DEVICE
+
+
+def test_missing_library_fails_loudly(tmp_path):
+    """No CPU fallback: with the CUDA library missing the binding raises."""
+    import subprocess, sys
+    code = ("import paper_conf_ipps_rockis11_b200 as pkg\n"
+            "try:\n    pkg.Mcts()\nexcept FileNotFoundError as e:\n    print('raised', e)\n")
+    env = dict(os.environ, MCTS_LIB=str(tmp_path / "missing.so"))
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=120,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert out.stdout.startswith("raised"), out.stdout + out.stderr
