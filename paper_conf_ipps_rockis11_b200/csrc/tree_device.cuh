@@ -18,6 +18,25 @@ namespace mcts_dev {
 
 constexpr u32 kNoChild = 0xFFFFFFFFu;
 constexpr int kMaxPath = 160;  // > 60 moves + passes + root
+
+// Debug build (MCTS_DEBUG_BOUNDS=1, tools/build_variants.py "bounds"): every
+// tree-slot index and path position is checked and a violation traps with the
+// line number printed — the stand-in for compute-sanitizer's memcheck, which
+// this GPU pool does not allow. Compiled out of the product build.
+#ifndef MCTS_DEBUG_BOUNDS
+#define MCTS_DEBUG_BOUNDS 0
+#endif
+#if MCTS_DEBUG_BOUNDS
+#define MCTS_CHECK(cond)                                                          \
+  do {                                                                             \
+    if (!(cond)) {                                                                 \
+      printf("MCTS_CHECK failed: %s (%s:%d)\n", #cond, __FILE__, __LINE__);      \
+      __trap();                                                                    \
+    }                                                                              \
+  } while (0)
+#else
+#define MCTS_CHECK(cond) do {} while (0)
+#endif
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
 struct TreePool {
@@ -176,6 +195,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
     u32 best_i = kNoChild, bm = 0, bf = 0, bk = 0, bw = 0, bd = 0;
     u64 bo = 0, bp = 0, bl = 0;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
+      MCTS_CHECK(first != kNoChild && first + i < T.slot_cap);
       const size_t c = base + first + i;
       const u32 wc = T.w[c], kc = T.k[c], dc = T.d[c], mc = T.meta[c], fc = T.first[c];
       u64 oc = 0, pc_ = 0, lc = 0;
@@ -200,6 +220,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
       lg = __shfl_sync(kFull, bl, src);
     }
     ++depth;
+    MCTS_CHECK(depth < kMaxPath && v < T.slot_cap);
     if (lane == 0) { pc->node[depth] = v; pc->k[depth] = kv; pc->w[depth] = wv; pc->d[depth] = dv; }
   }
   // Expansion (L179-L182), lane 0: the lowest-index untried move, or the pass
@@ -237,6 +258,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
         const u64 f = flips_loop(sq, own, opp, __brevll(own), __brevll(opp), rays);
         cown = opp & ~f; copp = own | f | (1ULL << sq); mv = (u32)sq;
       }
+      MCTS_CHECK(c < T.slot_cap && nch < limit && depth + 1 < kMaxPath);
       term = meta_term(init_node(T, base + c, cown, copp, mv, true)) ? 1u : 0u;
       T.meta[base + v] = meta + 1u;  // ++nchild
       if (depth == 0) { pc->root_meta = meta + 1u; pc->root_first = f0; }
@@ -263,6 +285,7 @@ __device__ __forceinline__ LeafInfo select_expand(const TreePool& T, size_t base
 __device__ __forceinline__ void backprop(const TreePool& T, size_t base, PathCache* pc, int depth,
                                          u32 W, u32 D, u32 Lo, int lane) {
   for (int p = lane; p <= depth; p += 32) {
+    MCTS_CHECK(pc->node[p] < T.slot_cap);
     const size_t s = base + pc->node[p];
     const int lvl = depth - p;
     const u32 k = pc->k[p] + 1u, w = pc->w[p] + ((lvl & 1) ? W : Lo), d = pc->d[p] + D;

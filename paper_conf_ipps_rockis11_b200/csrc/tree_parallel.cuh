@@ -155,6 +155,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
           __threadfence();  // acquire: v's board was published before its meta
           const u64 own = __ldcg(&T.own[v]), opp = __ldcg(&T.opp[v]), lg = __ldcg(&T.legal[v]);
           const u32 c = first + claimed;
+          MCTS_CHECK(c < T.slot_cap && depth + 1 < kMaxPath);
           if (lg == 0ULL) {
             tree_init_node(T, S, c, opp, own, 64u, 1u);  // pass: same discs, turn swaps
           } else {
@@ -180,6 +181,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
     u32 best_i = kNoChild, best_meta = 0, best_first = kNoChild, best_k = 0;
     for (u32 i = (u32)lane; i < nch; i += 32u) {
       const u32 c = first + i;
+      MCTS_CHECK(c < T.slot_cap);
       const u32 mc = ld_rlx(&T.meta[c]);
       const u32 kc = ld_rlx(&T.k[c]), vc = ld_rlx(&T.vl[c]), wc = ld_rlx(&T.w[c]);
       const u32 fc = ld_rlx(&T.first[c]);
@@ -199,6 +201,7 @@ __device__ __forceinline__ LeafInfo tree_select_expand(const TreePool& T, TreeSy
     kp = __shfl_sync(kFull, best_k, src);  // v's k + vl, read before our own virtual visit
     ++depth;
     if (lane == 0) {
+      MCTS_CHECK(depth < kMaxPath && v < T.slot_cap);
       path[depth] = v;
       atomicAdd(&T.vl[v], 1u);
     }

@@ -31,6 +31,7 @@ VARIANTS = {
     "t128m11": ["MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=11"],
     "t64m20": ["MCTS_PLAYOUT_THREADS=64", "MCTS_PLAYOUT_MINB=20"],
     "leafprobe": ["MCTS_LEAF_PROBE=1"],
+    "bounds": ["MCTS_DEBUG_BOUNDS=1"],
     "pair": ["MCTS_PAIR=1"],
     "pair_m3": ["MCTS_PAIR=1", "MCTS_PLAYOUT_MINB=3"],
     "pair_t128m5": ["MCTS_PAIR=1", "MCTS_PLAYOUT_THREADS=128", "MCTS_PLAYOUT_MINB=5"],
