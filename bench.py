@@ -37,7 +37,7 @@ sys.path.insert(0, ROOT)
 N_LEAVES, N_PER_LEAF, GEN_SEED, LMIN, LMAX = 4096, 256, 2, 20, 40
 OPEN_LMIN, OPEN_LMAX = 0, 8  # the opening-phase batch
 PLAYOUT_SEED = 2
-SEARCH_GATE_CYCLES = 100_000_000  # ~50 ms at the 1965 MHz SM clock (torch.cuda._sleep)
+SEARCH_GATE_CYCLES = 500_000_000  # ~250 ms at the 1965 MHz SM clock (torch.cuda._sleep)
 SEARCH_TREES, SEARCH_THREADS, SEARCH_MS = 1184, 128, 500.0
 LEAF_THREADS = 16384
 # (n_trees, threads_per_tree) of each scheme's searcher; for "tree" n_trees is
@@ -794,9 +794,11 @@ def main():
         torch.cuda.synchronize()
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        # a ~50 ms spin kernel ahead of e0 holds the stream while the host
+        # a ~250 ms spin kernel ahead of e0 holds the stream while the host
         # validates and enqueues the search, so the events bracket device work
-        # only (r2x / r2zb saw 12 / 49 ms host-side gaps inside the window)
+        # only (r2x / r2zb / r2zp saw 12 / 49 / 35 ms host-side gaps inside the
+        # window, r2zp behind a 50 ms gate: host CUDA calls stalled while the
+        # nvidia-smi clock sampler ran)
         with torch.cuda.stream(stream):
             torch.cuda._sleep(SEARCH_GATE_CYCLES)
         e0.record(stream)
