@@ -3,7 +3,8 @@
 Bar: bit-exact for everything — W/D/L counts, ply counts,
 generated positions, the ln table, and the full UCT root statistics and best
 move in iteration mode (the UCB arithmetic is correctly rounded IEEE double on
-both sides). Time mode is checked by invariants only (parity unpinned).
+both sides). Time mode stops on a wall-clock deadline, so how many iterations
+run is not reproducible: it is checked by invariants that hold at any count.
 """
 import numpy as np
 import pytest
